@@ -1,0 +1,175 @@
+/*
+ * kcore.h -- C ABI of the B200-native k-core decomposition library
+ *            (paper_conf_icde_ahmady0gcz23_b200/lib/libkcore.so).
+ *
+ * Problem (Sec. I; Sec. II-A): given an undirected
+ * simple graph G=(V,E), compute core(v) for every v, where the k-core is the
+ * largest induced subgraph of minimum degree >= k and core(v) is the largest
+ * k whose k-core contains v.  Input is CSR with dense vertex ids (P:L151-159,
+ * Sec. IV "Graph Organization in GPU"); output is core(v) for all v
+ * (Alg. 1 Input/Output).
+ *
+ * Method: level-synchronous degree-based peeling (the two-phase scan/loop
+ * framework of PKC/ParK that the paper follows, Alg. 1-3
+ * P:L187-298), re-designed for sm_100a as ONE persistent cooperative kernel
+ * per call: deg init (Alg. 1 l.1), level scan (Alg. 2) fused with the
+ * min-degree reduction for level skipping, peel sub-rounds (Alg. 3 l.12-24:
+ * atomicSub returning the old value, append on old == k+1, restore on
+ * old <= k, P:L322-334 / Fig. 6), with no host round-trip between levels or
+ * sub-rounds.  See DESIGN.md.
+ *
+ * Conventions shared by every entry point
+ *  - n      : |V|, 0 <= n < 2^31 (vertex ids are int32).
+ *  - m      : number of ARCS = 2|E| = rowptr[n] (NOT |E|; reading R3),
+ *             0 <= m < 2^33.
+ *  - rowptr : int64[n+1], rowptr[0] = 0, non-decreasing, rowptr[n] = m.
+ *  - colidx : int32[m]; row v lists N(v) strictly increasing (no duplicates),
+ *             no self-loops, and the arc set is symmetric (directed
+ *             inputs are made undirected by ignoring direction, reading R2).
+ *             These preconditions are NOT checked on the fast path; call
+ *             kcore_validate_csr() (tests/debug) to check them.
+ *  - core_out: int32[n] output; it also serves as the degree work array
+ *             (deg[] becomes core[] in place).
+ *  - Ownership: the caller owns all inputs/outputs; inputs are never
+ *             modified; the library never frees caller memory.  Scratch
+ *             (kcore_workspace_size bytes) is either caller-provided via
+ *             kcore_options.workspace or allocated stream-ordered
+ *             (cudaMallocAsync on `stream`) and freed before return.
+ *  - Streams: device entry points are stream-ordered; results are valid once
+ *             `stream` completes (no host synchronisation unless stats are
+ *             requested).  `stream` is a cudaStream_t (0 = legacy default).
+ *  - Errors : every function returns a kcore_status.  Argument errors are
+ *             reported before any launch and leave outputs untouched.
+ */
+#ifndef KCORE_H
+#define KCORE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    KCORE_OK = 0,
+    KCORE_EINVAL = -1,      /* bad argument (null pointer, n or m out of range)     */
+    KCORE_ENOMEM = -2,      /* device or host allocation failed                     */
+    KCORE_ECUDA = -3,       /* CUDA launch / runtime error                          */
+    KCORE_ENCCL = -4,       /* NCCL error (multi-GPU entry points)                  */
+    KCORE_EGRAPH = -5,      /* only from kcore_validate_csr: input violates the CSR */
+                            /* preconditions above                                  */
+    KCORE_EUNSUPPORTED = -6 /* device cannot run the kernel (e.g. not sm_100)       */
+} kcore_status;
+
+/* Algorithms selectable through kcore_options.algo. */
+#define KCORE_ALGO_PERSISTENT 0 /* default: one persistent kernel, device-resident loop */
+#define KCORE_ALGO_HOSTLOOP 1   /* ablation: paper Alg. 1 style host-driven loop of      */
+                                /* scan/peel launches (host round-trip per sub-round)   */
+
+typedef struct {
+    int32_t algo;            /* KCORE_ALGO_*                                           */
+    int32_t blocks_per_sm;   /* 0 = auto (occupancy); persistent grid = SMs x this     */
+    int32_t solo_arcs;       /* 0 = default; peel phases with fewer arcs run on one CTA */
+                             /* (no grid barrier); -1 disables the single-CTA path      */
+    int32_t reserved0;
+    int32_t *order_out;      /* optional DEVICE int32[n]: peel order (concatenated      */
+                             /* frontiers; a degeneracy order)          */
+    void *workspace;         /* optional DEVICE scratch of >= kcore_workspace_size()    */
+    size_t workspace_bytes;
+    int64_t reserved[4];
+} kcore_options;
+
+/* Run statistics (filled when a non-NULL pointer is passed; this makes the
+ * call synchronise `stream`). */
+typedef struct {
+    int64_t levels;        /* distinct core values peeled (levels scanned)            */
+    int64_t subrounds;     /* peel sub-rounds executed (grid-wide + single-CTA)        */
+    int64_t solo_subrounds;/* of which ran on a single CTA                             */
+    int64_t barriers;      /* grid barriers executed                                   */
+    int64_t scanned;       /* sum over levels of scanned entries (Sigma A_l)           */
+    int64_t arcs_walked;   /* arcs walked by the peel (= m for a full run)            */
+    int64_t compactions;   /* alive-list rewrites                                      */
+    int32_t kmax;          /* largest core number                                     */
+    int32_t grid_blocks;   /* persistent grid size                                     */
+    int32_t block_threads;
+    int32_t reserved0;
+    double kernel_ms;      /* device time of the decomposition kernel(s) (CUDA events) */
+    int64_t reserved[4];
+} kcore_stats;
+
+/* Core decomposition on one GPU (north-star signature).  All array pointers
+ * are DEVICE pointers.  Equivalent to kcore_decompose_ex(..., NULL, NULL). */
+int kcore_decompose(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                    int32_t *core_out, void *stream);
+
+/* Same, with options (may be NULL) and statistics (may be NULL). */
+int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                       int32_t *core_out, void *stream, const kcore_options *opt,
+                       kcore_stats *stats);
+
+/* End-to-end variant on HOST buffers: copies rowptr/colidx host->device,
+ * decomposes, copies core_out device->host, and synchronises `stream` before
+ * returning.  Host buffers should be pinned for full PCIe bandwidth.
+ * Device memory for the graph and scratch is allocated stream-ordered and
+ * freed before return. */
+int kcore_decompose_host(const int64_t *rowptr_host, const int32_t *colidx_host, int64_t n,
+                         int64_t m, int32_t *core_out_host, void *stream,
+                         const kcore_options *opt, kcore_stats *stats);
+
+/* Scratch bytes needed by kcore_decompose_ex for a graph with n vertices and
+ * m arcs (about 20 n bytes + 4 KiB). */
+size_t kcore_workspace_size(int64_t n, int64_t m);
+
+/* Check the CSR preconditions on the device (DEVICE pointers): rowptr[0]==0,
+ * monotone, rowptr[n]==m, ids in range, no self-loops, rows strictly
+ * increasing, symmetric.  Returns KCORE_OK, KCORE_EGRAPH, or an error.
+ * Synchronises `stream`. */
+int kcore_validate_csr(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                       void *stream);
+
+/* Human-readable name of a status code (static string). */
+const char *kcore_strerror(int status);
+
+/* Library version string. */
+const char *kcore_version(void);
+
+/* ---------------------------------------------------------------------------
+ * Multi-GPU: 1D vertex-range ownership (north star; the paper's multi-GPU
+ * future work, with owner routing instead of a master GPU).
+ * Rank r owns vertices [v_begin, v_end) and stores their rows:
+ *   rowptr_local int64[v_end-v_begin+1] (local offsets, rowptr_local[0]=0),
+ *   colidx_local int32[m_local] with GLOBAL neighbour ids,
+ *   core_out_local int32[v_end-v_begin].
+ * Ranges must tile [0, n_global) in rank order (rank 0 starts at 0).
+ * Per peel sub-round every rank peels its owned frontier, applies local
+ * decrements in place and routes remote ones to their owners with one NCCL
+ * all-to-all; an all-reduce of {frontier non-empty, min next degree} ends
+ * sub-rounds and levels.  Host-driven: synchronises `stream` once per
+ * sub-round.  All ranks must call collectively.
+ * ------------------------------------------------------------------------- */
+int kcore_decompose_mg(const int64_t *rowptr_local, const int32_t *colidx_local,
+                       int64_t n_global, int64_t v_begin, int64_t v_end, int64_t m_local,
+                       int32_t *core_out_local, void *stream, void *nccl_comm,
+                       kcore_stats *stats);
+
+/* The same protocol with `nranks` VIRTUAL ranks on the current device and a
+ * device-memory loopback transport in place of NCCL (same kernels, same
+ * driver, same routing).  Takes the GLOBAL CSR (DEVICE pointers), partitions
+ * it into equal vertex ranges internally and writes the global core_out.  For
+ * testing the multi-GPU protocol on one GPU.  Synchronises `stream`. */
+int kcore_decompose_mg_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n,
+                               int64_t m, int32_t nranks, int32_t *core_out, void *stream,
+                               kcore_stats *stats);
+
+/* NCCL plumbing for callers without their own communicator (the Python
+ * binding uses these; the unique id is exchanged over torch.distributed).
+ * kcore_nccl_unique_id writes 128 bytes.  The comm handle is an ncclComm_t. */
+int kcore_nccl_unique_id(void *id_out_128);
+int kcore_nccl_comm_init(void **comm_out, int32_t nranks, const void *id_128, int32_t rank);
+int kcore_nccl_comm_destroy(void *comm);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* KCORE_H */

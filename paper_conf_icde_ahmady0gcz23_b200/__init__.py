@@ -1,0 +1,255 @@
+"""B200-native k-core decomposition (Ahmad et al., ICDE 2023 -- PAPER.md).
+
+Thin Python binding over the C ABI in ``include/kcore.h`` (library
+``lib/libkcore.so``, built in-tree by ``make``).  Argument marshalling only:
+every step of the decomposition runs in the library's sm_100a kernels.  PyTorch
+supplies device memory, streams and process groups.  There is no CPU fallback:
+if the library is missing or the device is not a B200 every call raises.
+
+Entry points mirror the C names:
+
+* :func:`kcore_decompose`       -- core numbers of a CSR graph on one GPU.
+* :func:`kcore_decompose_host`  -- same from/to host buffers (end-to-end path).
+* :func:`kcore_decompose_mg`    -- multi-GPU, 1-D vertex-range ownership (NCCL).
+* :func:`kcore_decompose_mg_virtual` -- the multi-GPU protocol with virtual
+  ranks on one GPU (testing).
+* :func:`kcore_validate_csr`, :func:`kcore_workspace_size`, :func:`kcore_strerror`.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "lib", "libkcore.so")
+
+KCORE_OK = 0
+KCORE_EINVAL = -1
+KCORE_ENOMEM = -2
+KCORE_ECUDA = -3
+KCORE_ENCCL = -4
+KCORE_EGRAPH = -5
+KCORE_EUNSUPPORTED = -6
+
+ALGO_PERSISTENT = 0
+ALGO_HOSTLOOP = 1
+
+# every symbol include/kcore.h declares (checked by tests/test_abi.py)
+EXPORTS = (
+    "kcore_decompose", "kcore_decompose_ex", "kcore_decompose_host", "kcore_workspace_size",
+    "kcore_validate_csr", "kcore_strerror", "kcore_version", "kcore_decompose_mg",
+    "kcore_decompose_mg_virtual", "kcore_nccl_unique_id", "kcore_nccl_comm_init",
+    "kcore_nccl_comm_destroy",
+)
+
+
+class KcoreError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        self.status = status
+        super().__init__(f"{what}: {strerror(status)} ({status})")
+
+
+class _Options(ctypes.Structure):
+    _fields_ = [
+        ("algo", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
+        ("solo_arcs", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+        ("order_out", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
+        ("workspace_bytes", ctypes.c_size_t), ("reserved", ctypes.c_int64 * 4),
+    ]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [
+        ("levels", ctypes.c_int64), ("subrounds", ctypes.c_int64),
+        ("solo_subrounds", ctypes.c_int64), ("barriers", ctypes.c_int64),
+        ("scanned", ctypes.c_int64), ("arcs_walked", ctypes.c_int64),
+        ("compactions", ctypes.c_int64), ("kmax", ctypes.c_int32),
+        ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
+        ("reserved0", ctypes.c_int32), ("kernel_ms", ctypes.c_double),
+        ("reserved", ctypes.c_int64 * 4),
+    ]
+
+
+@dataclass
+class Stats:
+    levels: int
+    subrounds: int
+    solo_subrounds: int
+    barriers: int
+    scanned: int
+    arcs_walked: int
+    compactions: int
+    kmax: int
+    grid_blocks: int
+    block_threads: int
+    kernel_ms: float
+
+    @classmethod
+    def _from(cls, s: _Stats) -> "Stats":
+        return cls(s.levels, s.subrounds, s.solo_subrounds, s.barriers, s.scanned, s.arcs_walked,
+                   s.compactions, s.kmax, s.grid_blocks, s.block_threads, s.kernel_ms)
+
+
+_lib = None
+
+
+def _load():
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: build it with `make` (__graft_entry__.build()); "
+                               "there is no CPU fallback")
+        import torch  # noqa: F401  (loads torch's libnccl.so.2 first so both share one copy)
+        lib = ctypes.CDLL(LIB_PATH)
+        vp, i64, i32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32
+        lib.kcore_decompose.argtypes = [vp, vp, i64, i64, vp, vp]
+        lib.kcore_decompose_ex.argtypes = [vp, vp, i64, i64, vp, vp, ctypes.POINTER(_Options),
+                                           ctypes.POINTER(_Stats)]
+        lib.kcore_decompose_host.argtypes = [vp, vp, i64, i64, vp, vp, ctypes.POINTER(_Options),
+                                             ctypes.POINTER(_Stats)]
+        lib.kcore_workspace_size.argtypes = [i64, i64]
+        lib.kcore_workspace_size.restype = ctypes.c_size_t
+        lib.kcore_validate_csr.argtypes = [vp, vp, i64, i64, vp]
+        lib.kcore_strerror.argtypes = [ctypes.c_int]
+        lib.kcore_strerror.restype = ctypes.c_char_p
+        lib.kcore_version.restype = ctypes.c_char_p
+        lib.kcore_decompose_mg.argtypes = [vp, vp, i64, i64, i64, i64, vp, vp, vp, ctypes.POINTER(_Stats)]
+        lib.kcore_decompose_mg_virtual.argtypes = [vp, vp, i64, i64, i32, vp, vp, ctypes.POINTER(_Stats)]
+        lib.kcore_nccl_unique_id.argtypes = [vp]
+        lib.kcore_nccl_comm_init.argtypes = [ctypes.POINTER(vp), i32, vp, i32]
+        lib.kcore_nccl_comm_destroy.argtypes = [vp]
+        _lib = lib
+    return _lib
+
+
+def library():
+    """The loaded ctypes handle (raises if the library is missing)."""
+    return _load()
+
+
+def strerror(status: int) -> str:
+    try:
+        return _load().kcore_strerror(status).decode()
+    except RuntimeError:
+        return f"status {status}"
+
+
+def version() -> str:
+    return _load().kcore_version().decode()
+
+
+def kcore_workspace_size(n: int, m: int = 0) -> int:
+    return int(_load().kcore_workspace_size(n, m))
+
+
+def _stream_ptr(device):
+    import torch
+    return torch.cuda.current_stream(device).cuda_stream
+
+
+def _check_csr_tensors(rowptr, colidx):
+    import torch
+    if not (rowptr.is_cuda and colidx.is_cuda):
+        raise ValueError("rowptr/colidx must be CUDA tensors (use kcore_decompose_host for host buffers)")
+    if rowptr.dtype != torch.int64 or colidx.dtype != torch.int32:
+        raise TypeError("rowptr must be int64 and colidx int32")
+    if not (rowptr.is_contiguous() and colidx.is_contiguous()):
+        raise ValueError("rowptr/colidx must be contiguous")
+    if rowptr.device != colidx.device:
+        raise ValueError("rowptr/colidx on different devices")
+
+
+def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=None,
+                    algo: int = ALGO_PERSISTENT, blocks_per_sm: int = 0, solo_arcs: int = 0,
+                    stats: bool = False):
+    """Core numbers of the graph (rowptr int64[n+1], colidx int32[m] CUDA tensors).
+
+    Runs on the current stream of the tensors' device.  Returns an int32 tensor
+    ``core`` (and a :class:`Stats` if ``stats=True``, which synchronises)."""
+    import torch
+    _check_csr_tensors(rowptr, colidx)
+    dev = rowptr.device
+    n = rowptr.numel() - 1
+    m = colidx.numel()
+    if core_out is None:
+        core_out = torch.empty(max(n, 0), dtype=torch.int32, device=dev)
+    opt = _Options(algo, blocks_per_sm, solo_arcs, 0,
+                   order_out.data_ptr() if order_out is not None else None,
+                   workspace.data_ptr() if workspace is not None else None,
+                   workspace.numel() * workspace.element_size() if workspace is not None else 0)
+    st = _Stats()
+    with torch.cuda.device(dev):
+        rc = _load().kcore_decompose_ex(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
+                                        core_out.data_ptr() if n else None, _stream_ptr(dev),
+                                        ctypes.byref(opt), ctypes.byref(st) if stats else None)
+    if rc != KCORE_OK:
+        raise KcoreError(rc, "kcore_decompose")
+    return (core_out, Stats._from(st)) if stats else core_out
+
+
+def kcore_decompose_host(rowptr, colidx, *, core_out=None, stats: bool = False, device=None,
+                         algo: int = ALGO_PERSISTENT):
+    """End-to-end: host (ideally pinned) int64/int32 tensors in, host int32 core out."""
+    import torch
+    if rowptr.is_cuda or colidx.is_cuda:
+        raise ValueError("kcore_decompose_host takes host tensors")
+    if rowptr.dtype != torch.int64 or colidx.dtype != torch.int32:
+        raise TypeError("rowptr must be int64 and colidx int32")
+    dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+    n = rowptr.numel() - 1
+    m = colidx.numel()
+    if core_out is None:
+        core_out = torch.empty(max(n, 0), dtype=torch.int32, pin_memory=rowptr.is_pinned())
+    opt = _Options(algo, 0, 0, 0, None, None, 0)
+    st = _Stats()
+    with torch.cuda.device(dev):
+        rc = _load().kcore_decompose_host(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
+                                          core_out.data_ptr() if n else None, _stream_ptr(dev),
+                                          ctypes.byref(opt), ctypes.byref(st) if stats else None)
+    if rc != KCORE_OK:
+        raise KcoreError(rc, "kcore_decompose_host")
+    return (core_out, Stats._from(st)) if stats else core_out
+
+
+def kcore_validate_csr(rowptr, colidx) -> int:
+    """KCORE_OK if the CUDA CSR satisfies the preconditions, else KCORE_EGRAPH."""
+    import torch
+    _check_csr_tensors(rowptr, colidx)
+    n = rowptr.numel() - 1
+    m = colidx.numel()
+    with torch.cuda.device(rowptr.device):
+        rc = _load().kcore_validate_csr(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
+                                        _stream_ptr(rowptr.device))
+    if rc not in (KCORE_OK, KCORE_EGRAPH):
+        raise KcoreError(rc, "kcore_validate_csr")
+    return rc
+
+
+def kcore_decompose_mg_virtual(rowptr, colidx, nranks: int, *, stats: bool = False):
+    """Multi-GPU protocol with `nranks` virtual ranks on this GPU (global CSR in, global core out)."""
+    import torch
+    _check_csr_tensors(rowptr, colidx)
+    dev = rowptr.device
+    n = rowptr.numel() - 1
+    m = colidx.numel()
+    core = torch.empty(max(n, 0), dtype=torch.int32, device=dev)
+    st = _Stats()
+    with torch.cuda.device(dev):
+        rc = _load().kcore_decompose_mg_virtual(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
+                                                nranks, core.data_ptr() if n else None, _stream_ptr(dev),
+                                                ctypes.byref(st) if stats else None)
+    if rc != KCORE_OK:
+        raise KcoreError(rc, "kcore_decompose_mg_virtual")
+    return (core, Stats._from(st)) if stats else core
+
+
+from .parallel import (  # noqa: E402
+    NcclComm, kcore_decompose_mg, owner_ranges, local_csr, gather_cores,
+)
+
+__all__ = [
+    "kcore_decompose", "kcore_decompose_host", "kcore_decompose_mg", "kcore_decompose_mg_virtual",
+    "kcore_validate_csr", "kcore_workspace_size", "strerror", "version", "Stats", "KcoreError",
+    "NcclComm", "owner_ranges", "local_csr", "gather_cores", "EXPORTS", "LIB_PATH",
+]

@@ -1,0 +1,72 @@
+// kc_common.cuh -- PTX helpers and launch constants shared by the sm_100a
+// kernels of the k-core hot path.  (Product code; shares nothing with oracle/.)
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace kc {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// 64-bit queue tail packs (#vertices appended << 33) | (#arcs appended) so one
+// atomicAdd reserves frontier slots and their arc range together.
+constexpr int kArcBits = 33;
+constexpr unsigned long long kArcMask = (1ULL << kArcBits) - 1ULL;
+constexpr unsigned long long kCntOne = 1ULL << kArcBits;
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void st_release_u32(uint32_t *p, uint32_t v)
+{
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ uint32_t atom_add_release_u32(uint32_t *p, uint32_t v)
+{
+    uint32_t old;
+    asm volatile("atom.release.gpu.global.add.u32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+    return old;
+}
+
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long *p)
+{
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ int32_t ld_relaxed_i32(const int32_t *p)
+{
+    int32_t v;
+    asm volatile("ld.relaxed.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// streaming read-only loads of the CSR (never written during a call)
+__device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p)
+{
+    int32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+
+__device__ __forceinline__ int64_t ld_ro_i64(const int64_t *p) { return __ldg(p); }
+
+// L2-coherent loads of data other CTAs write during the call (deg, queue)
+__device__ __forceinline__ int32_t ld_cg_i32(const int32_t *p) { return __ldcg(p); }
+__device__ __forceinline__ int64_t ld_cg_i64(const int64_t *p) { return __ldcg(p); }
+
+__device__ __forceinline__ unsigned lanemask_lt()
+{
+    unsigned m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+} // namespace kc

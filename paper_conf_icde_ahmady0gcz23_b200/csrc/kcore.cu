@@ -1,0 +1,318 @@
+// kcore.cu -- C ABI of the single-GPU hot path (include/kcore.h).
+//
+// kcore_decompose_ex: validate arguments, carve the workspace, initialise the
+// device State, then launch ONE persistent cooperative kernel (k_persistent)
+// that runs deg init, every level scan, every peel sub-round and the level
+// control on the device (see kc_kernels.cuh).  The ablation KCORE_ALGO_HOSTLOOP
+// drives the same phase code from the host like the paper's Alg. 1
+// (P:L187-208): one launch per phase and a device->host read-back after each.
+#include "kcore.h"
+#include "kc_kernels.cuh"
+
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+
+using namespace kc;
+
+namespace {
+
+constexpr int kMaxDev = 64;
+
+struct DevInfo {
+    int sms = 0;
+    int occ = 0;  // resident CTAs of k_persistent per SM
+    int major = 0, minor = 0;
+    bool init = false;
+};
+
+DevInfo g_dev[kMaxDev];
+std::mutex g_mu;
+
+int dev_info(DevInfo &out)
+{
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return KCORE_ECUDA;
+    if (dev < 0 || dev >= kMaxDev) return KCORE_ECUDA;
+    std::lock_guard<std::mutex> lk(g_mu);
+    DevInfo &d = g_dev[dev];
+    if (!d.init) {
+        if (cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess)
+            return KCORE_ECUDA;
+        cudaDeviceGetAttribute(&d.major, cudaDevAttrComputeCapabilityMajor, dev);
+        cudaDeviceGetAttribute(&d.minor, cudaDevAttrComputeCapabilityMinor, dev);
+        if (d.major != 10) return KCORE_EUNSUPPORTED;
+        int occ = 0;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_persistent, kBlock, 0) != cudaSuccess)
+            return KCORE_ECUDA;
+        d.occ = occ;
+        d.init = true;
+    }
+    out = d;
+    return KCORE_OK;
+}
+
+size_t al(size_t x) { return (x + 255) & ~(size_t)255; }
+
+struct Carve {
+    State *S;
+    int32_t *order;
+    int64_t *qarc;
+    int32_t *alive0, *alive1;
+};
+
+size_t carve(void *base, int64_t n, Carve *c)
+{
+    size_t off = 0;
+    auto take = [&](size_t bytes) {
+        char *p = base ? (char *)base + off : nullptr;
+        off += al(bytes);
+        return p;
+    };
+    Carve t;
+    t.S = (State *)take(sizeof(State));
+    t.order = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    t.qarc = (int64_t *)take(sizeof(int64_t) * (size_t)(n + 1));
+    t.alive0 = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    t.alive1 = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    if (c) *c = t;
+    return off;
+}
+
+int check_args(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+               const int32_t *core_out)
+{
+    if (n < 0 || n >= ((int64_t)1 << 31)) return KCORE_EINVAL;
+    if (m < 0 || m >= ((int64_t)1 << kArcBits)) return KCORE_EINVAL;
+    if (n > 0 && (!rowptr || !core_out)) return KCORE_EINVAL;
+    if (m > 0 && !colidx) return KCORE_EINVAL;
+    if (n == 0 && m != 0) return KCORE_EINVAL;
+    return KCORE_OK;
+}
+
+int default_solo_arcs() { return 16384; }
+
+} // namespace
+
+#define KC_CUDA(x)                                                                                 \
+    do {                                                                                           \
+        cudaError_t e_ = (x);                                                                      \
+        if (e_ != cudaSuccess) {                                                                   \
+            rc = (e_ == cudaErrorMemoryAllocation) ? KCORE_ENOMEM : KCORE_ECUDA;                   \
+            goto done;                                                                             \
+        }                                                                                          \
+    } while (0)
+
+extern "C" size_t kcore_workspace_size(int64_t n, int64_t m)
+{
+    (void)m;
+    if (n < 0) return 0;
+    return carve(nullptr, n, nullptr);
+}
+
+extern "C" const char *kcore_strerror(int status)
+{
+    switch (status) {
+    case KCORE_OK: return "KCORE_OK";
+    case KCORE_EINVAL: return "KCORE_EINVAL: invalid argument";
+    case KCORE_ENOMEM: return "KCORE_ENOMEM: allocation failed";
+    case KCORE_ECUDA: return "KCORE_ECUDA: CUDA error";
+    case KCORE_ENCCL: return "KCORE_ENCCL: NCCL error";
+    case KCORE_EGRAPH: return "KCORE_EGRAPH: CSR violates the preconditions";
+    case KCORE_EUNSUPPORTED: return "KCORE_EUNSUPPORTED: device is not sm_100";
+    default: return "KCORE: unknown status";
+    }
+}
+
+extern "C" const char *kcore_version(void) { return "kcore-b200 0.1 (sm_100a persistent peel)"; }
+
+extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, int64_t n,
+                                  int64_t m, int32_t *core_out, void *stream_,
+                                  const kcore_options *opt, kcore_stats *stats)
+{
+    int rc = check_args(rowptr, colidx, n, m, core_out);
+    if (rc) return rc;
+    if (stats) memset(stats, 0, sizeof(*stats));
+    if (n == 0) return KCORE_OK;
+    cudaStream_t st = (cudaStream_t)stream_;
+    DevInfo di;
+    rc = dev_info(di);
+    if (rc) return rc;
+
+    const int algo = opt ? opt->algo : KCORE_ALGO_PERSISTENT;
+    if (algo != KCORE_ALGO_PERSISTENT && algo != KCORE_ALGO_HOSTLOOP) return KCORE_EINVAL;
+    int bps = (opt && opt->blocks_per_sm > 0) ? opt->blocks_per_sm : di.occ;
+    if (bps > di.occ) bps = di.occ;
+    if (bps < 1) return KCORE_EUNSUPPORTED;
+    const int grid = di.sms * bps;
+    int solo = default_solo_arcs();
+    if (opt && opt->solo_arcs > 0) solo = opt->solo_arcs;
+    if (opt && opt->solo_arcs < 0) solo = 0;
+
+    const size_t need = carve(nullptr, n, nullptr);
+    void *ws = nullptr;
+    bool own_ws = false;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    int32_t *d_phase = nullptr;
+    State hS;
+    Carve cv;
+    KArgs A;
+    if (opt && opt->workspace) {
+        if (opt->workspace_bytes < need) return KCORE_EINVAL;
+        ws = opt->workspace;
+    } else {
+        KC_CUDA(cudaMallocAsync(&ws, need, st));
+        own_ws = true;
+    }
+    carve(ws, n, &cv);
+    A.rowptr = rowptr;
+    A.colidx = colidx;
+    A.deg = core_out;
+    A.order = cv.order;
+    A.qarc = cv.qarc;
+    A.alive[0] = cv.alive0;
+    A.alive[1] = cv.alive1;
+    A.S = cv.S;
+    A.n = n;
+
+    if (stats) {
+        KC_CUDA(cudaEventCreate(&ev0));
+        KC_CUDA(cudaEventCreate(&ev1));
+    }
+    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, grid);
+    KC_CUDA(cudaGetLastError());
+    if (stats) KC_CUDA(cudaEventRecord(ev0, st));
+    if (algo == KCORE_ALGO_PERSISTENT) {
+        void *args[] = {&A};
+        KC_CUDA(cudaLaunchCooperativeKernel((const void *)k_persistent, dim3(grid), dim3(kBlock), args,
+                                            0, st));
+    } else {
+        KC_CUDA(cudaMallocAsync((void **)&d_phase, sizeof(int32_t), st));
+        int32_t ph = PH_INIT;
+        int guard = 0;
+        while (ph != PH_DONE) {
+            k_phase<<<grid, kBlock, 0, st>>>(A);
+            k_leader<<<1, 1, 0, st>>>(A, d_phase);
+            KC_CUDA(cudaGetLastError());
+            KC_CUDA(cudaMemcpyAsync(&ph, d_phase, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+            KC_CUDA(cudaStreamSynchronize(st));
+            if (++guard > (1 << 28)) { rc = KCORE_ECUDA; goto done; }
+        }
+    }
+    if (stats) KC_CUDA(cudaEventRecord(ev1, st));
+    if (opt && opt->order_out)
+        KC_CUDA(cudaMemcpyAsync(opt->order_out, cv.order, sizeof(int32_t) * (size_t)n,
+                                cudaMemcpyDeviceToDevice, st));
+    if (stats) {
+        KC_CUDA(cudaMemcpyAsync(&hS, cv.S, sizeof(State), cudaMemcpyDeviceToHost, st));
+        KC_CUDA(cudaStreamSynchronize(st));
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, ev0, ev1);
+        stats->levels = hS.st_levels;
+        stats->subrounds = hS.st_subrounds;
+        stats->solo_subrounds = hS.st_solo_subrounds;
+        stats->barriers = hS.st_barriers;
+        stats->scanned = hS.st_scanned;
+        stats->arcs_walked = hS.st_arcs;
+        stats->compactions = hS.st_compactions;
+        stats->kmax = hS.st_kmax;
+        stats->grid_blocks = grid;
+        stats->block_threads = kBlock;
+        stats->kernel_ms = ms;
+    }
+done:
+    if (d_phase) cudaFreeAsync(d_phase, st);
+    if (own_ws && ws) cudaFreeAsync(ws, st);
+    if (ev0) cudaEventDestroy(ev0);
+    if (ev1) cudaEventDestroy(ev1);
+    return rc;
+}
+
+extern "C" int kcore_decompose(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                               int32_t *core_out, void *stream)
+{
+    return kcore_decompose_ex(rowptr, colidx, n, m, core_out, stream, nullptr, nullptr);
+}
+
+extern "C" int kcore_decompose_host(const int64_t *rowptr_h, const int32_t *colidx_h, int64_t n,
+                                    int64_t m, int32_t *core_h, void *stream_,
+                                    const kcore_options *opt, kcore_stats *stats)
+{
+    int rc = check_args(rowptr_h, colidx_h, n, m, core_h);
+    if (rc) return rc;
+    if (n == 0) {
+        if (stats) memset(stats, 0, sizeof(*stats));
+        return KCORE_OK;
+    }
+    cudaStream_t st = (cudaStream_t)stream_;
+    int64_t *d_rp = nullptr;
+    int32_t *d_ci = nullptr, *d_core = nullptr;
+    KC_CUDA(cudaMallocAsync((void **)&d_rp, sizeof(int64_t) * (size_t)(n + 1), st));
+    KC_CUDA(cudaMallocAsync((void **)&d_ci, sizeof(int32_t) * (size_t)(m > 0 ? m : 1), st));
+    KC_CUDA(cudaMallocAsync((void **)&d_core, sizeof(int32_t) * (size_t)n, st));
+    KC_CUDA(cudaMemcpyAsync(d_rp, rowptr_h, sizeof(int64_t) * (size_t)(n + 1), cudaMemcpyHostToDevice, st));
+    if (m > 0)
+        KC_CUDA(cudaMemcpyAsync(d_ci, colidx_h, sizeof(int32_t) * (size_t)m, cudaMemcpyHostToDevice, st));
+    rc = kcore_decompose_ex(d_rp, d_ci, n, m, d_core, st, opt, stats);
+    if (rc) goto done;
+    KC_CUDA(cudaMemcpyAsync(core_h, d_core, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToHost, st));
+    KC_CUDA(cudaStreamSynchronize(st));
+done:
+    if (d_rp) cudaFreeAsync(d_rp, st);
+    if (d_ci) cudaFreeAsync(d_ci, st);
+    if (d_core) cudaFreeAsync(d_core, st);
+    if (cudaStreamSynchronize(st) != cudaSuccess && rc == KCORE_OK) rc = KCORE_ECUDA;
+    return rc;
+}
+
+// ------------------------------------------------------------ validation
+namespace {
+__global__ void k_validate(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                           int *flag)
+{
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (tid == 0 && (rowptr[0] != 0 || rowptr[n] != m)) atomicOr(flag, 1);
+    for (int64_t v = tid; v < n; v += stride) {
+        const int64_t b = rowptr[v], e = rowptr[v + 1];
+        if (e < b || b < 0 || e > m) { atomicOr(flag, 1); continue; }
+        int32_t prev = -1;
+        for (int64_t x = b; x < e; x++) {
+            const int32_t u = colidx[x];
+            if (u < 0 || u >= n) { atomicOr(flag, 2); break; }
+            if (u == v) { atomicOr(flag, 4); break; }
+            if (u <= prev) { atomicOr(flag, 8); break; }
+            prev = u;
+            // symmetric: v must appear in N(u)
+            int64_t lo = rowptr[u], hi = rowptr[u + 1];
+            if (lo < 0 || hi > m || hi < lo) { atomicOr(flag, 1); break; }
+            while (lo < hi) {
+                const int64_t mid = lo + (hi - lo) / 2;
+                if (colidx[mid] < (int32_t)v) lo = mid + 1; else hi = mid;
+            }
+            if (lo >= rowptr[u + 1] || colidx[lo] != (int32_t)v) { atomicOr(flag, 16); break; }
+        }
+    }
+}
+} // namespace
+
+extern "C" int kcore_validate_csr(const int64_t *rowptr, const int32_t *colidx, int64_t n,
+                                  int64_t m, void *stream_)
+{
+    int rc = check_args(rowptr, colidx, n, m, (const int32_t *)rowptr);
+    if (rc) return rc;
+    if (n == 0) return KCORE_OK;
+    cudaStream_t st = (cudaStream_t)stream_;
+    int *d_flag = nullptr, h_flag = 0;
+    KC_CUDA(cudaMallocAsync((void **)&d_flag, sizeof(int), st));
+    KC_CUDA(cudaMemsetAsync(d_flag, 0, sizeof(int), st));
+    k_validate<<<1184, 256, 0, st>>>(rowptr, colidx, n, m, d_flag);
+    KC_CUDA(cudaGetLastError());
+    KC_CUDA(cudaMemcpyAsync(&h_flag, d_flag, sizeof(int), cudaMemcpyDeviceToHost, st));
+    KC_CUDA(cudaStreamSynchronize(st));
+    rc = h_flag ? KCORE_EGRAPH : KCORE_OK;
+done:
+    if (d_flag) cudaFreeAsync(d_flag, st);
+    cudaStreamSynchronize(st);
+    return rc;
+}
