@@ -70,14 +70,20 @@ typedef enum {
 typedef struct {
     int32_t algo;            /* KCORE_ALGO_*                                           */
     int32_t blocks_per_sm;   /* 0 = auto (occupancy); persistent grid = SMs x this     */
-    int32_t solo_arcs;       /* 0 = default; peel phases with fewer arcs run on one CTA */
-                             /* (no grid barrier); -1 disables the single-CTA path      */
-    int32_t reserved0;
+    int32_t solo_arcs;       /* 0 = default; peel sub-rounds with <= this many arcs run */
+                             /* on ONE CTA with CTA-local sync (no grid barrier); -1 off */
+    int32_t solo_scan;       /* 0 = default; level scans over <= this many alive       */
+                             /* entries run on one CTA; -1 off                          */
     int32_t *order_out;      /* optional DEVICE int32[n]: peel order (concatenated      */
                              /* frontiers; a degeneracy order)          */
     void *workspace;         /* optional DEVICE scratch of >= kcore_workspace_size()    */
     size_t workspace_bytes;
-    int64_t reserved[4];
+    int64_t *trace_out;      /* optional DEVICE int64[trace_cap][8]: one record per     */
+                             /* phase {globaltimer ns, clock64, phase<<8|solo<<4|grid,  */
+                             /* k, frontier or scan length, arcs, queue count, 0}       */
+    int64_t trace_cap;       /* records available at trace_out (records written are     */
+                             /* reported in kcore_stats.trace_len)                      */
+    int64_t reserved[3];
 } kcore_options;
 
 /* Run statistics (filled when a non-NULL pointer is passed; this makes the
@@ -93,7 +99,7 @@ typedef struct {
     int32_t kmax;          /* largest core number                                     */
     int32_t grid_blocks;   /* persistent grid size                                     */
     int32_t block_threads;
-    int32_t reserved0;
+    int32_t trace_len;     /* trace records written (see kcore_options.trace_out)    */
     double kernel_ms;      /* device time of the decomposition kernel(s) (CUDA events) */
     int64_t reserved[4];
 } kcore_stats;

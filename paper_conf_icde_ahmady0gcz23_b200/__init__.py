@@ -53,9 +53,10 @@ class KcoreError(RuntimeError):
 class _Options(ctypes.Structure):
     _fields_ = [
         ("algo", ctypes.c_int32), ("blocks_per_sm", ctypes.c_int32),
-        ("solo_arcs", ctypes.c_int32), ("reserved0", ctypes.c_int32),
+        ("solo_arcs", ctypes.c_int32), ("solo_scan", ctypes.c_int32),
         ("order_out", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
-        ("workspace_bytes", ctypes.c_size_t), ("reserved", ctypes.c_int64 * 4),
+        ("workspace_bytes", ctypes.c_size_t), ("trace_out", ctypes.c_void_p),
+        ("trace_cap", ctypes.c_int64), ("reserved", ctypes.c_int64 * 3),
     ]
 
 
@@ -66,7 +67,7 @@ class _Stats(ctypes.Structure):
         ("scanned", ctypes.c_int64), ("arcs_walked", ctypes.c_int64),
         ("compactions", ctypes.c_int64), ("kmax", ctypes.c_int32),
         ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
-        ("reserved0", ctypes.c_int32), ("kernel_ms", ctypes.c_double),
+        ("trace_len", ctypes.c_int32), ("kernel_ms", ctypes.c_double),
         ("reserved", ctypes.c_int64 * 4),
     ]
 
@@ -84,11 +85,12 @@ class Stats:
     grid_blocks: int
     block_threads: int
     kernel_ms: float
+    trace_len: int = 0
 
     @classmethod
     def _from(cls, s: _Stats) -> "Stats":
         return cls(s.levels, s.subrounds, s.solo_subrounds, s.barriers, s.scanned, s.arcs_walked,
-                   s.compactions, s.kmax, s.grid_blocks, s.block_threads, s.kernel_ms)
+                   s.compactions, s.kmax, s.grid_blocks, s.block_threads, s.kernel_ms, s.trace_len)
 
 
 _lib = None
@@ -162,7 +164,7 @@ def _check_csr_tensors(rowptr, colidx):
 
 def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=None,
                     algo: int = ALGO_PERSISTENT, blocks_per_sm: int = 0, solo_arcs: int = 0,
-                    stats: bool = False):
+                    solo_scan: int = 0, trace=None, stats: bool = False):
     """Core numbers of the graph (rowptr int64[n+1], colidx int32[m] CUDA tensors).
 
     Runs on the current stream of the tensors' device.  Returns an int32 tensor
@@ -174,10 +176,12 @@ def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=
     m = colidx.numel()
     if core_out is None:
         core_out = torch.empty(max(n, 0), dtype=torch.int32, device=dev)
-    opt = _Options(algo, blocks_per_sm, solo_arcs, 0,
+    opt = _Options(algo, blocks_per_sm, solo_arcs, solo_scan,
                    order_out.data_ptr() if order_out is not None else None,
                    workspace.data_ptr() if workspace is not None else None,
-                   workspace.numel() * workspace.element_size() if workspace is not None else 0)
+                   workspace.numel() * workspace.element_size() if workspace is not None else 0,
+                   trace.data_ptr() if trace is not None else None,
+                   trace.shape[0] if trace is not None else 0)
     st = _Stats()
     with torch.cuda.device(dev):
         rc = _load().kcore_decompose_ex(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
@@ -201,7 +205,7 @@ def kcore_decompose_host(rowptr, colidx, *, core_out=None, stats: bool = False, 
     m = colidx.numel()
     if core_out is None:
         core_out = torch.empty(max(n, 0), dtype=torch.int32, pin_memory=rowptr.is_pinned())
-    opt = _Options(algo, 0, 0, 0, None, None, 0)
+    opt = _Options(algo, 0, 0, 0, None, None, 0, None, 0)
     st = _Stats()
     with torch.cuda.device(dev):
         rc = _load().kcore_decompose_host(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,

@@ -5,27 +5,31 @@
 //
 //   INIT   deg[v] = rowptr[v+1]-rowptr[v] into core_out, min-degree reduce    (Alg.1 l.1)
 //   SCAN   level k: frontier <- {v alive : deg[v] == k}; fused min{deg > k};   (Alg.2)
-//          optional alive-list compaction (reading R6 / Q14)
+//          optional alive-list compaction (reading R6)
 //   PEEL   sub-round over frontier slots [s,e): for every arc (v,u):          (Alg.3 l.12-24)
 //          if deg[u] > k: old = atomicSub(&deg[u],1);
 //             old == k+1 -> append u (it reached k: next sub-round)
 //             old <= k   -> atomicAdd(&deg[u],1)  (restore, Fig. 6)
 //             else       -> min_next = min(min_next, old-1)   (level skip, reading R5)
-//   SOLO   a small peel sub-round sequence run by ONE CTA with __syncthreads
-//          instead of grid barriers (latency path for tiny frontiers)
 //   level end: k <- max(k+1, min_next)  (Alg.1 l.9 does k+1; reading R5)
 //
-// Phases are separated by a grid barrier whose last arriver ("leader") runs
-// the level/sub-round control logic (Alg.1 l.5-9 and Alg.3 l.5) on the device
-// and publishes the next phase, so there is no host round-trip at all.
+// Control.  Every CTA keeps an identical copy of the control state (Ctrl) in
+// shared memory.  A phase ends with a grid barrier whose last arriver takes a
+// SNAPSHOT of the three counters (queue tail, compaction length, min) and
+// resets them; every CTA then advances its Ctrl with the same pure function
+// advance(Ctrl, Snap).  No host round-trip, no serial "leader" logic.
+// Phases whose work is tiny (a few thousand arcs, or a short alive list) are
+// marked `solo`: CTA 0 runs them -- and every following tiny phase, across
+// sub-rounds and levels -- alone with __syncthreads instead of grid barriers,
+// then publishes its Ctrl; the other CTAs wait at one barrier.
 //
-// The frontier queue is one array order[n] (every vertex is appended exactly
-// once in the whole run, so it cannot overflow -- cf. the paper's per-block
-// buf[i] and ring buffers) plus qarc[n]: the exclusive prefix
-// of the appended vertices' degrees.  A packed 64-bit tail (count<<33 | arcs)
-// reserves slots and their arc range with one atomic, so a peel sub-round can
-// split its ARCS evenly over all warps (hub vertices are shared by many warps;
-// no degree buckets needed).
+// Frontier queue: one array order[n] (every vertex is appended exactly once in
+// the whole run, so it cannot overflow -- cf. the paper's per-block buf[i] and
+// ring buffers) plus qarc[n], the exclusive prefix of the
+// appended vertices' degrees.  A packed 64-bit tail (count<<33 | arcs)
+// reserves slots and their arc range with one atomic, so a peel sub-round
+// splits its ARCS evenly over all warps (hubs are shared by many warps; no
+// degree buckets needed).
 #pragma once
 
 #include "kc_common.cuh"
@@ -40,37 +44,45 @@ constexpr int kScanTile = kBlock * kScanItems;
 constexpr int kStageCap = 256;  // per-warp append stage (>= 32 * kUnroll)
 constexpr int kUnroll = 4;      // arcs per lane in flight per peel batch
 constexpr int kBatch = 32 * kUnroll;
+constexpr int kTraceFields = 8;
 
-enum : int32_t { PH_INIT = 0, PH_SCAN = 1, PH_PEEL = 2, PH_SOLO = 3, PH_DONE = 4 };
+enum : int32_t { PH_INIT = 0, PH_SCAN = 1, PH_PEEL = 2, PH_DONE = 3 };
 
-struct Ctl {
-    int32_t phase, k, level, compact;
-    int32_t src_sel, dst_sel, solo_block, pad;
-    int64_t src_len;
-    int64_t s, e, as, ae;  // PEEL/SOLO: slots [s,e), arcs [as,ae)
+// Control state; replicated in every CTA, advanced by advance().
+struct Ctrl {
+    int32_t phase, solo, k, level_min;
+    int32_t compact, src_sel, dst_sel, alive_sel;
+    int64_t src_len, alive_len;
+    int64_t s, e, as, ae;         // PEEL: slots [s,e), arcs [as,ae)
+    int64_t lvl_cnt0, lvl_arc0;   // queue tail when the level's scan began
+    int64_t st_levels, st_sub, st_solo_sub, st_bar, st_scanned, st_arcs, st_compact;
+    int32_t st_kmax, st_pad;
 };
 
-struct alignas(128) State {
-    unsigned long long qtail;      // packed (count << 33) | arcs
-    unsigned long long alive_out;  // compaction output length
-    int32_t min_next;              // atomicMin target for the level skip
-    uint32_t bar_count;            // grid barrier arrivals (monotone)
-    uint32_t bar_gen;              // grid barrier generation
-    int32_t nblocks;
-    Ctl ctl[2];                    // published by the leader, indexed by gen & 1
-    // leader-private bookkeeping
+struct Snap {
+    unsigned long long qtail, alive_out;
+    int32_t min;
+    int32_t pad;
+};
+
+struct Params {
     int64_t n;
-    int64_t lvl_cnt0, lvl_arc0;    // queue tail when the current level's scan began
-    int64_t alive_len;
-    int32_t alive_sel;             // -1: no alive list yet (scan the identity)
-    int32_t solo_arcs;             // peel phases with <= this many arcs go SOLO
-    int64_t solo_e, solo_ae;       // progress reported by a SOLO phase
-    int64_t solo_sub;              // sub-rounds run by the SOLO phase
-    // statistics
-    int64_t st_levels, st_subrounds, st_solo_subrounds, st_barriers, st_scanned, st_arcs,
-        st_compactions;
-    int32_t st_kmax;
-    int32_t error;
+    int32_t solo_arcs;  // PEEL phases with <= this many arcs run solo
+    int32_t solo_scan;  // SCAN phases over <= this many entries run solo
+};
+
+struct State {
+    alignas(128) unsigned long long qtail;      // packed (count << 33) | arcs
+    alignas(128) unsigned long long alive_out;  // compaction output length
+    alignas(128) int32_t min_next;              // atomicMin target
+    alignas(128) uint32_t bar_count;            // grid barrier arrivals (monotone)
+    alignas(128) uint32_t bar_gen;              // grid barrier generation
+    Snap snap[2];                               // counters at barrier gen, by gen & 1
+    alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
+    alignas(128) Params prm;
+    int64_t *trace;                             // optional [trace_cap][kTraceFields]
+    int64_t trace_cap;
+    unsigned long long trace_n;
 };
 
 struct KArgs {
@@ -92,9 +104,8 @@ struct Smem {
     unsigned long long tot_q, base_q;
     unsigned long long tot_k, base_k;
     int32_t red_min[kWarps];
-    Ctl ctl;
-    uint32_t gen;
-    int32_t solo_go;
+    Ctrl ctrl;
+    Snap snap;
 };
 
 // ---------------------------------------------------------------- helpers
@@ -110,6 +121,13 @@ __device__ __forceinline__ int64_t warp_sum64(int64_t v)
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
     return v;
+}
+
+__device__ __forceinline__ unsigned long long globaltimer()
+{
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
 }
 
 // CTA-wide min, then one atomicMin per CTA
@@ -227,7 +245,7 @@ __device__ __forceinline__ void block_scan2(Smem &sm, unsigned long long q, uint
     k_ex = sm.scan_k[wib] + (ki - kk);
 }
 
-__device__ void phase_scan(const KArgs &A, const Ctl &c, Smem &sm)
+__device__ void phase_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
 {
     const int k = c.k;
     const int32_t *src = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
@@ -235,7 +253,7 @@ __device__ void phase_scan(const KArgs &A, const Ctl &c, Smem &sm)
     const int64_t len = c.src_len;
     const int64_t ntiles = (len + kScanTile - 1) / kScanTile;
     int lmin = INT_MAX;
-    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (int64_t t = bid; t < ntiles; t += nblk) {
         int32_t vv[kScanItems], dd[kScanItems], fd[kScanItems];
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
@@ -306,7 +324,7 @@ __device__ __forceinline__ int64_t find_slot(const int64_t *qarc, int64_t s, int
     return lo + (31 - __clz(b));
 }
 
-// Walk arcs [a0,a1) of the frontier [s,e) (arc range [as,ae)) with one warp.
+// Walk arcs [a0,a1) of the frontier [s,e) (arc range [.,ae)) with one warp.
 __device__ __forceinline__ void peel_range(const KArgs &A, Smem &sm, const int k, int64_t s,
                                            int64_t e, int64_t ae, int64_t a0, int64_t a1,
                                            int &scnt, int &lmin)
@@ -372,11 +390,11 @@ __device__ __forceinline__ void peel_range(const KArgs &A, Smem &sm, const int k
     }
 }
 
-__device__ void phase_peel(const KArgs &A, const Ctl &c, Smem &sm)
+__device__ void phase_peel(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
 {
     const int wib = threadIdx.x >> 5;
-    const int64_t gw = (int64_t)blockIdx.x * kWarps + wib;
-    const int64_t W = (int64_t)gridDim.x * kWarps;
+    const int64_t gw = (int64_t)bid * kWarps + wib;
+    const int64_t W = (int64_t)nblk * kWarps;
     const int64_t T = c.ae - c.as;
     int64_t C = (T + W - 1) / W;
     C = ((C + kBatch - 1) / kBatch) * kBatch;
@@ -387,147 +405,101 @@ __device__ void phase_peel(const KArgs &A, const Ctl &c, Smem &sm)
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
-// SOLO: this CTA alone runs sub-rounds starting at [s,e) until the frontier
-// is empty or grows past the solo threshold; reports progress in the State.
-__device__ void phase_solo(const KArgs &A, const Ctl &c, Smem &sm)
-{
-    const int wib = threadIdx.x >> 5;
-    int64_t s = c.s, e = c.e, as = c.as, ae = c.ae, sub = 0;
-    int lmin = INT_MAX;
-    while (true) {
-        const int64_t T = ae - as;
-        int64_t C = (T + kWarps - 1) / kWarps;
-        C = ((C + kBatch - 1) / kBatch) * kBatch;
-        int scnt = 0;
-        const int64_t a0 = as + (int64_t)wib * C;
-        if (a0 < ae) peel_range(A, sm, c.k, s, e, ae, a0, min(a0 + C, ae), scnt, lmin);
-        warp_flush(A, sm, wib, scnt);
-        sub++;
-        __threadfence();
-        __syncthreads();
-        if (threadIdx.x == 0) sm.base_q = ld_relaxed_u64(&A.S->qtail);
-        __syncthreads();
-        const unsigned long long qt = sm.base_q;
-        const int64_t cnt = (int64_t)(qt >> kArcBits), arcs = (int64_t)(qt & kArcMask);
-        __syncthreads();
-        s = e; as = ae; e = cnt; ae = arcs;
-        if (e == s || ae == as || (ae - as) > (int64_t)A.S->solo_arcs) break;
-    }
-    block_min_atomic(sm, lmin, &A.S->min_next);
-    if (threadIdx.x == 0) {
-        volatile State *S = A.S;
-        S->solo_e = s;   // first slot NOT yet peeled
-        S->solo_ae = as;
-        S->solo_sub = sub;
-    }
-}
-
 // ---------------------------------------------------------------- control
-// Runs on ONE thread (the last CTA to arrive at a barrier) while every other
-// CTA waits: reads the counters and publishes the next phase in ctl[(gen+1)&1].
-__device__ __noinline__ void leader_step(const KArgs &A, uint32_t gen)
+// The pure transition function (Alg.1 l.5-9, Alg.3 l.5 and the level skip).
+// Every CTA applies it to identical inputs, so all copies stay identical.
+__device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
 {
-    volatile State *S = A.S;
-    Ctl cur;
-    {
-        volatile Ctl *pc = &S->ctl[gen & 1];
-        cur.phase = pc->phase; cur.k = pc->k; cur.level = pc->level; cur.compact = pc->compact;
-        cur.src_sel = pc->src_sel; cur.dst_sel = pc->dst_sel; cur.solo_block = pc->solo_block;
-        cur.pad = 0; cur.src_len = pc->src_len;
-        cur.s = pc->s; cur.e = pc->e; cur.as = pc->as; cur.ae = pc->ae;
-    }
-    Ctl nx = cur;
-    const unsigned long long qt = ld_relaxed_u64(&A.S->qtail);
-    const int64_t cnt = (int64_t)(qt >> kArcBits), arcs = (int64_t)(qt & kArcMask);
-    const int64_t n = S->n;
-    S->st_barriers = S->st_barriers + 1;
-
-    bool level_end = false;
-    int64_t ps = 0, pe = 0, pas = 0, pae = 0;  // next peel frontier, if any
-    bool peel = false;
-    switch (cur.phase) {
-    case PH_INIT: {
-        const int k0 = ld_relaxed_i32(&A.S->min_next);
-        S->min_next = INT_MAX;
-        nx.level = -1;
-        nx.k = (k0 == INT_MAX) ? 0 : k0;
-        break;
-    }
-    case PH_SCAN: {
-        if (cur.compact) {
-            S->alive_sel = cur.dst_sel;
-            S->alive_len = (int64_t)ld_relaxed_u64(&A.S->alive_out);
-            S->st_compactions = S->st_compactions + 1;
+    const int64_t cnt = (int64_t)(sn.qtail >> kArcBits), arcs = (int64_t)(sn.qtail & kArcMask);
+    c.level_min = min(c.level_min, sn.min);
+    bool level_end = false, peel = false;
+    int64_t ps = 0, pe = 0, pas = 0, pae = 0;
+    int next_k = 0;
+    if (c.phase == PH_INIT) {
+        next_k = (c.level_min == INT_MAX) ? 0 : c.level_min;
+        c.level_min = INT_MAX;
+    } else if (c.phase == PH_SCAN) {
+        c.st_scanned += c.src_len;
+        if (c.compact) {
+            c.alive_sel = c.dst_sel;
+            c.alive_len = (int64_t)sn.alive_out;
+            c.st_compact++;
         }
-        S->st_scanned = S->st_scanned + cur.src_len;
-        const int64_t c0 = S->lvl_cnt0, a0 = S->lvl_arc0;
-        if (arcs > a0) { peel = true; ps = c0; pe = cnt; pas = a0; pae = arcs; }
+        if (arcs > c.lvl_arc0) { peel = true; ps = c.lvl_cnt0; pe = cnt; pas = c.lvl_arc0; pae = arcs; }
         else level_end = true;
-        break;
-    }
-    case PH_PEEL: {
-        S->st_subrounds = S->st_subrounds + 1;
-        S->st_arcs = S->st_arcs + (cur.ae - cur.as);
-        if (cnt > cur.e && arcs > cur.ae) { peel = true; ps = cur.e; pe = cnt; pas = cur.ae; pae = arcs; }
+    } else if (c.phase == PH_PEEL) {
+        c.st_sub++;
+        if (c.solo) c.st_solo_sub++;
+        c.st_arcs += c.ae - c.as;
+        if (cnt > c.e && arcs > c.ae) { peel = true; ps = c.e; pe = cnt; pas = c.ae; pae = arcs; }
         else level_end = true;
-        break;
     }
-    case PH_SOLO: {
-        S->st_subrounds = S->st_subrounds + S->solo_sub;
-        S->st_solo_subrounds = S->st_solo_subrounds + S->solo_sub;
-        S->st_arcs = S->st_arcs + (S->solo_ae - cur.as);
-        const int64_t se = S->solo_e, sae = S->solo_ae;
-        if (cnt > se && arcs > sae) { peel = true; ps = se; pe = cnt; pas = sae; pae = arcs; }
-        else level_end = true;
-        break;
-    }
-    default: break;
-    }
-
-    int next_k = nx.k;
-    bool start_scan = (cur.phase == PH_INIT);
+    bool scan = (c.phase == PH_INIT);
     if (level_end) {
-        S->st_levels = S->st_levels + 1;
-        S->st_kmax = cur.k;
-        if (cnt >= n) {
-            nx.phase = PH_DONE;
+        if (cnt > c.lvl_cnt0) { c.st_levels++; c.st_kmax = c.k; }
+        if (cnt >= p.n) {
+            c.phase = PH_DONE;
+            c.solo = 0;
         } else {
-            const int mn = ld_relaxed_i32(&A.S->min_next);
-            S->min_next = INT_MAX;
-            next_k = max(cur.k + 1, mn);
-            start_scan = true;
+            next_k = max(c.k + 1, c.level_min);
+            c.level_min = INT_MAX;
+            scan = true;
         }
     }
     if (peel) {
-        const bool solo = S->solo_arcs > 0 && (pae - pas) <= (int64_t)S->solo_arcs;
-        nx.phase = solo ? PH_SOLO : PH_PEEL;
-        nx.solo_block = -1;
-        nx.s = ps; nx.e = pe; nx.as = pas; nx.ae = pae;
-    } else if (start_scan) {
-        const int64_t live = n - cnt;
-        const int src_sel = S->alive_sel;
-        const int64_t src_len = src_sel < 0 ? n : S->alive_len;
-        const bool compact = src_sel < 0 ? (live * 4 < n) : (live * 2 < src_len);
-        nx.phase = PH_SCAN;
-        nx.k = next_k;
-        nx.level = nx.level + 1;
-        nx.src_sel = src_sel;
-        nx.src_len = src_len;
-        nx.compact = compact ? 1 : 0;
-        nx.dst_sel = src_sel < 0 ? 0 : 1 - src_sel;
-        if (compact) S->alive_out = 0;
-        S->lvl_cnt0 = cnt;
-        S->lvl_arc0 = arcs;
+        c.phase = PH_PEEL;
+        c.solo = (pae - pas) <= (int64_t)p.solo_arcs;
+        c.s = ps; c.e = pe; c.as = pas; c.ae = pae;
+    } else if (scan) {
+        const int64_t live = p.n - cnt;
+        const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
+        const bool compact = c.alive_sel < 0 ? (live * 4 < p.n) : (live * 2 < src_len);
+        c.phase = PH_SCAN;
+        c.k = next_k;
+        c.src_sel = c.alive_sel;
+        c.src_len = src_len;
+        c.compact = compact ? 1 : 0;
+        c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
+        c.solo = src_len <= (int64_t)p.solo_scan;
+        c.lvl_cnt0 = cnt;
+        c.lvl_arc0 = arcs;
     }
-    volatile Ctl *pn = &S->ctl[(gen + 1) & 1];
-    pn->phase = nx.phase; pn->k = nx.k; pn->level = nx.level; pn->compact = nx.compact;
-    pn->src_sel = nx.src_sel; pn->dst_sel = nx.dst_sel; pn->solo_block = nx.solo_block;
-    pn->src_len = nx.src_len; pn->s = nx.s; pn->e = nx.e; pn->as = nx.as; pn->ae = nx.ae;
 }
 
-// Grid barrier; the last arriver runs leader_step before releasing.  Copies
-// the published Ctl into shared memory.  Returns whether this CTA was leader.
-__device__ __forceinline__ bool grid_sync(const KArgs &A, Smem &sm)
+// Snapshot + reset of the counters (caller guarantees nobody else touches them).
+__device__ __forceinline__ Snap take_snapshot(State *S)
+{
+    Snap sn;
+    sn.qtail = ld_relaxed_u64(&S->qtail);
+    sn.alive_out = ld_relaxed_u64(&S->alive_out);
+    sn.min = ld_relaxed_i32(&S->min_next);
+    sn.pad = 0;
+    S->alive_out = 0ULL;
+    S->min_next = INT_MAX;
+    return sn;
+}
+
+__device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &sn, int grid)
+{
+    if (!S->trace) return;
+    const unsigned long long i = S->trace_n;
+    if ((int64_t)i >= S->trace_cap) return;
+    int64_t *r = S->trace + i * kTraceFields;
+    r[0] = (int64_t)globaltimer();
+    r[1] = (int64_t)clock64();
+    r[2] = ((int64_t)c.phase << 8) | ((int64_t)c.solo << 4) | grid;  // phase that ENDED
+    r[3] = c.k;
+    r[4] = c.phase == PH_SCAN ? c.src_len : (c.e - c.s);
+    r[5] = c.phase == PH_PEEL ? (c.ae - c.as) : 0;
+    r[6] = (int64_t)(sn.qtail >> kArcBits);
+    r[7] = 0;
+    S->trace_n = i + 1;
+}
+
+// Grid barrier; the last arriver snapshots+resets the counters.  Leaves the
+// snapshot in sm.snap (thread 0 only is guaranteed to see it before the final
+// __syncthreads; all threads after).
+__device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
 {
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -535,86 +507,150 @@ __device__ __forceinline__ bool grid_sync(const KArgs &A, Smem &sm)
         const uint32_t gen = ld_acquire_u32(&S->bar_gen);
         __threadfence();
         const uint32_t t = atom_add_release_u32(&S->bar_count, 1u);
-        const bool last = (t + 1u) == (uint32_t)gridDim.x * (gen + 1u);
-        if (last) {
+        Snap sn;
+        if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
             __threadfence();
-            leader_step(A, gen);
-            __threadfence();
+            sn = take_snapshot(S);
+            S->snap[(gen + 1u) & 1u] = sn;
             st_release_u32(&S->bar_gen, gen + 1u);
         } else {
             while (ld_acquire_u32(&S->bar_gen) == gen) {
             }
+            const Snap *ps = &S->snap[(gen + 1u) & 1u];
+            sn.qtail = ld_relaxed_u64(&ps->qtail);
+            sn.alive_out = ld_relaxed_u64(&ps->alive_out);
+            sn.min = ld_relaxed_i32(&ps->min);
+            sn.pad = 0;
         }
-        volatile Ctl *pc = &S->ctl[(gen + 1u) & 1u];
-        sm.ctl.phase = pc->phase; sm.ctl.k = pc->k; sm.ctl.level = pc->level;
-        sm.ctl.compact = pc->compact; sm.ctl.src_sel = pc->src_sel; sm.ctl.dst_sel = pc->dst_sel;
-        sm.ctl.solo_block = pc->solo_block; sm.ctl.src_len = pc->src_len;
-        sm.ctl.s = pc->s; sm.ctl.e = pc->e; sm.ctl.as = pc->as; sm.ctl.ae = pc->ae;
-        sm.gen = gen + 1u;
-        sm.solo_go = last;
+        sm.snap = sn;
     }
     __syncthreads();
-    return sm.solo_go != 0;
+}
+
+__device__ __forceinline__ void run_phase(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+{
+    if (c.phase == PH_SCAN) phase_scan(A, c, sm, bid, nblk);
+    else if (c.phase == PH_PEEL) phase_peel(A, c, sm, bid, nblk);
+}
+
+// CTA 0 alone: run consecutive solo phases with CTA-local synchronisation.
+__device__ void solo_run(const KArgs &A, Smem &sm, const Params &p)
+{
+    State *S = A.S;
+    while (true) {
+        const Ctrl c = sm.ctrl;
+        run_phase(A, c, sm, 0, 1);  // ends with __syncthreads (block_min_atomic)
+        if (threadIdx.x == 0) {
+            __threadfence();
+            const Snap sn = take_snapshot(S);
+            trace_rec(S, sm.ctrl, sn, 0);
+            advance(sm.ctrl, sn, p);
+        }
+        __syncthreads();
+        if (sm.ctrl.phase == PH_DONE || !sm.ctrl.solo) break;
+    }
+    if (threadIdx.x == 0) {
+        S->pub = sm.ctrl;
+        __threadfence();
+    }
 }
 
 __global__ void __launch_bounds__(kBlock, 2) k_persistent(KArgs A)
 {
     __shared__ Smem sm;
-    phase_init(A, sm);
-    bool leader = grid_sync(A, sm);
-    while (true) {
-        const Ctl c = sm.ctl;
-        if (c.phase == PH_DONE) break;
-        if (c.phase == PH_SCAN) phase_scan(A, c, sm);
-        else if (c.phase == PH_PEEL) phase_peel(A, c, sm);
-        else if (c.phase == PH_SOLO) { if (leader) phase_solo(A, c, sm); }
-        leader = grid_sync(A, sm);
+    State *S = A.S;
+    const Params p = S->prm;
+    if (threadIdx.x == 0) {
+        Ctrl z = {};
+        z.phase = PH_INIT;
+        z.level_min = INT_MAX;
+        z.alive_sel = -1;
+        z.src_sel = -1;
+        sm.ctrl = z;
     }
+    phase_init(A, sm);
+    grid_barrier(A, sm);
+    if (threadIdx.x == 0) advance(sm.ctrl, sm.snap, p);
+    __syncthreads();
+    while (true) {
+        if (sm.ctrl.phase == PH_DONE) break;
+        if (sm.ctrl.solo) {
+            if (blockIdx.x == 0) solo_run(A, sm, p);
+            grid_barrier(A, sm);
+            if (threadIdx.x == 0) {
+                const Ctrl *pc = &S->pub;
+                Ctrl c;
+                // plain loads are safe: written before CTA 0's release-arrive,
+                // read after this CTA's acquire; bypass L1 with ld.cg
+                const int4 *src = reinterpret_cast<const int4 *>(pc);
+                int4 *dst = reinterpret_cast<int4 *>(&c);
+#pragma unroll
+                for (int w = 0; w < (int)(sizeof(Ctrl) / sizeof(int4)); w++) dst[w] = __ldcg(src + w);
+                c.st_bar++;
+                sm.ctrl = c;
+            }
+        } else {
+            const Ctrl c = sm.ctrl;
+            run_phase(A, c, sm, blockIdx.x, gridDim.x);
+            grid_barrier(A, sm);
+            if (threadIdx.x == 0) {
+                if (blockIdx.x == 0) trace_rec(S, sm.ctrl, sm.snap, 1);
+                sm.ctrl.st_bar++;
+                advance(sm.ctrl, sm.snap, p);
+            }
+        }
+        __syncthreads();
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) S->pub = sm.ctrl;  // final statistics
 }
 
 // -------------------------------------------- host-driven ablation kernels
-// (KCORE_ALGO_HOSTLOOP: paper Alg. 1 structure, one launch per phase plus a
-// host read-back of the phase.)
+// (KCORE_ALGO_HOSTLOOP: the paper's Alg. 1 structure -- one launch per phase
+// and a host read-back of the phase after each.  No solo phases.)
 __global__ void __launch_bounds__(kBlock, 2) k_phase(KArgs A)
 {
     __shared__ Smem sm;
-    if (threadIdx.x == 0) {
-        volatile State *S = A.S;
-        volatile Ctl *pc = &S->ctl[S->bar_gen & 1u];
-        sm.ctl.phase = pc->phase; sm.ctl.k = pc->k; sm.ctl.level = pc->level;
-        sm.ctl.compact = pc->compact; sm.ctl.src_sel = pc->src_sel; sm.ctl.dst_sel = pc->dst_sel;
-        sm.ctl.solo_block = pc->solo_block; sm.ctl.src_len = pc->src_len;
-        sm.ctl.s = pc->s; sm.ctl.e = pc->e; sm.ctl.as = pc->as; sm.ctl.ae = pc->ae;
-    }
+    if (threadIdx.x == 0) sm.ctrl = A.S->pub;
     __syncthreads();
-    const Ctl c = sm.ctl;
+    const Ctrl c = sm.ctrl;
     if (c.phase == PH_INIT) phase_init(A, sm);
-    else if (c.phase == PH_SCAN) phase_scan(A, c, sm);
-    else if (c.phase == PH_PEEL) phase_peel(A, c, sm);
-    else if (c.phase == PH_SOLO) { if (blockIdx.x == 0) phase_solo(A, c, sm); }
+    else run_phase(A, c, sm, blockIdx.x, gridDim.x);
 }
 
 __global__ void k_leader(KArgs A, int32_t *phase_out)
 {
     State *S = A.S;
-    const uint32_t gen = S->bar_gen;
-    leader_step(A, gen);
-    S->bar_gen = gen + 1u;
-    *phase_out = S->ctl[(gen + 1u) & 1u].phase;
+    const Params p = S->prm;
+    Ctrl c = S->pub;
+    const Snap sn = take_snapshot(S);
+    trace_rec(S, c, sn, 1);
+    c.st_bar++;
+    advance(c, sn, p);
+    S->pub = c;
+    *phase_out = c.phase;
 }
 
-__global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t nblocks)
+__global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan,
+                             int64_t *trace, int64_t trace_cap)
 {
     if (threadIdx.x == 0 && blockIdx.x == 0) {
-        State z = {};
-        z.min_next = INT_MAX;
-        z.nblocks = nblocks;
-        z.ctl[0].phase = PH_INIT;
-        z.ctl[1].phase = PH_INIT;
-        z.n = n;
+        S->qtail = 0ULL;
+        S->alive_out = 0ULL;
+        S->min_next = INT_MAX;
+        S->bar_count = 0u;
+        S->bar_gen = 0u;
+        Ctrl z = {};
+        z.phase = PH_INIT;
+        z.level_min = INT_MAX;
         z.alive_sel = -1;
-        z.solo_arcs = solo_arcs;
-        *S = z;
+        z.src_sel = -1;
+        S->pub = z;
+        S->prm.n = n;
+        S->prm.solo_arcs = solo_arcs;
+        S->prm.solo_scan = solo_scan;
+        S->trace = trace;
+        S->trace_cap = trace ? trace_cap : 0;
+        S->trace_n = 0ULL;
     }
 }
 

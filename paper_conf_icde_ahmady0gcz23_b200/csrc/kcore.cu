@@ -91,6 +91,7 @@ int check_args(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t 
 }
 
 int default_solo_arcs() { return 16384; }
+int default_solo_scan() { return 32768; }
 
 } // namespace
 
@@ -145,9 +146,14 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     if (bps > di.occ) bps = di.occ;
     if (bps < 1) return KCORE_EUNSUPPORTED;
     const int grid = di.sms * bps;
-    int solo = default_solo_arcs();
+    int solo = default_solo_arcs(), solo_scan = default_solo_scan();
     if (opt && opt->solo_arcs > 0) solo = opt->solo_arcs;
     if (opt && opt->solo_arcs < 0) solo = 0;
+    if (opt && opt->solo_scan > 0) solo_scan = opt->solo_scan;
+    if (opt && opt->solo_scan < 0) solo_scan = 0;
+    if (algo == KCORE_ALGO_HOSTLOOP) solo = solo_scan = 0;
+    int64_t *trace = opt ? opt->trace_out : nullptr;
+    const int64_t trace_cap = (opt && opt->trace_out) ? opt->trace_cap : 0;
 
     const size_t need = carve(nullptr, n, nullptr);
     void *ws = nullptr;
@@ -179,7 +185,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaEventCreate(&ev0));
         KC_CUDA(cudaEventCreate(&ev1));
     }
-    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, grid);
+    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, trace, trace_cap);
     KC_CUDA(cudaGetLastError());
     if (stats) KC_CUDA(cudaEventRecord(ev0, st));
     if (algo == KCORE_ALGO_PERSISTENT) {
@@ -208,16 +214,18 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaStreamSynchronize(st));
         float ms = 0.f;
         cudaEventElapsedTime(&ms, ev0, ev1);
-        stats->levels = hS.st_levels;
-        stats->subrounds = hS.st_subrounds;
-        stats->solo_subrounds = hS.st_solo_subrounds;
-        stats->barriers = hS.st_barriers;
-        stats->scanned = hS.st_scanned;
-        stats->arcs_walked = hS.st_arcs;
-        stats->compactions = hS.st_compactions;
-        stats->kmax = hS.st_kmax;
-        stats->grid_blocks = grid;
+        const Ctrl &c = hS.pub;
+        stats->levels = c.st_levels;
+        stats->subrounds = c.st_sub;
+        stats->solo_subrounds = c.st_solo_sub;
+        stats->barriers = c.st_bar;
+        stats->scanned = c.st_scanned;
+        stats->arcs_walked = c.st_arcs;
+        stats->compactions = c.st_compact;
+        stats->kmax = c.st_kmax;
+        stats->grid_blocks = algo == KCORE_ALGO_PERSISTENT ? grid : grid;
         stats->block_threads = kBlock;
+        stats->trace_len = (int32_t)hS.trace_n;
         stats->kernel_ms = ms;
     }
 done:

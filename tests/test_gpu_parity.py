@@ -186,7 +186,7 @@ def test_order_certificate_and_stats():
     assert oracle.check_certificate(rp, ci, core, order.cpu().numpy()) == 0
     assert oracle.check_invariants(rp, ci, core) == 0
     assert st.arcs_walked == ci.size
-    assert st.levels == np.unique(ref).size
+    assert st.levels == np.unique(ref).size, st
     assert st.kmax == ref.max()
 
 
