@@ -62,6 +62,9 @@ typedef enum {
     KCORE_EUNSUPPORTED = -6 /* device cannot run the kernel (e.g. not sm_100)       */
 } kcore_status;
 
+/* kcore_options.flags */
+#define KCORE_FLAG_NO_BLOOM 1   /* disable the shared-memory alive-set filter (ablation) */
+
 /* Algorithms selectable through kcore_options.algo. */
 #define KCORE_ALGO_PERSISTENT 0 /* default: one persistent kernel, device-resident loop */
 #define KCORE_ALGO_HOSTLOOP 1   /* ablation: paper Alg. 1 style host-driven loop of      */
@@ -83,25 +86,28 @@ typedef struct {
                              /* k, frontier or scan length, arcs, queue count, 0}       */
     int64_t trace_cap;       /* records available at trace_out (records written are     */
                              /* reported in kcore_stats.trace_len)                      */
-    int64_t reserved[3];
+    int32_t flags;           /* KCORE_FLAG_* bits                                        */
+    int32_t reserved1;
+    int64_t reserved[2];
 } kcore_options;
 
 /* Run statistics (filled when a non-NULL pointer is passed; this makes the
  * call synchronise `stream`). */
 typedef struct {
-    int64_t levels;        /* distinct core values peeled (levels scanned)            */
-    int64_t subrounds;     /* peel sub-rounds executed (grid-wide + single-CTA)        */
-    int64_t solo_subrounds;/* of which ran on a single CTA                             */
+    int64_t levels;        /* distinct core values peeled (non-empty levels)          */
+    int64_t phases;        /* LEVEL + HUB phases executed (grid-wide or single-CTA)   */
+    int64_t solo_phases;   /* of which ran on a single CTA                             */
     int64_t barriers;      /* grid barriers executed                                   */
     int64_t scanned;       /* sum over levels of scanned entries (Sigma A_l)           */
     int64_t arcs_walked;   /* arcs walked by the peel (= m for a full run)            */
     int64_t compactions;   /* alive-list rewrites                                      */
+    int64_t hub_arcs;      /* arcs walked in grid-wide (global queue) HUB phases       */
     int32_t kmax;          /* largest core number                                     */
     int32_t grid_blocks;   /* persistent grid size                                     */
     int32_t block_threads;
     int32_t trace_len;     /* trace records written (see kcore_options.trace_out)    */
     double kernel_ms;      /* device time of the decomposition kernel(s) (CUDA events) */
-    int64_t reserved[4];
+    int64_t reserved[3];
 } kcore_stats;
 
 /* Core decomposition on one GPU (north-star signature).  All array pointers
@@ -124,7 +130,7 @@ int kcore_decompose_host(const int64_t *rowptr_host, const int32_t *colidx_host,
                          const kcore_options *opt, kcore_stats *stats);
 
 /* Scratch bytes needed by kcore_decompose_ex for a graph with n vertices and
- * m arcs (about 20 n bytes + 4 KiB). */
+ * m arcs (about 36 n bytes + 4 KiB). */
 size_t kcore_workspace_size(int64_t n, int64_t m);
 
 /* Check the CSR preconditions on the device (DEVICE pointers): rowptr[0]==0,

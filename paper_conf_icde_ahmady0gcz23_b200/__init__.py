@@ -56,31 +56,33 @@ class _Options(ctypes.Structure):
         ("solo_arcs", ctypes.c_int32), ("solo_scan", ctypes.c_int32),
         ("order_out", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
         ("workspace_bytes", ctypes.c_size_t), ("trace_out", ctypes.c_void_p),
-        ("trace_cap", ctypes.c_int64), ("reserved", ctypes.c_int64 * 3),
+        ("trace_cap", ctypes.c_int64), ("flags", ctypes.c_int32), ("reserved1", ctypes.c_int32),
+        ("reserved", ctypes.c_int64 * 2),
     ]
 
 
 class _Stats(ctypes.Structure):
     _fields_ = [
-        ("levels", ctypes.c_int64), ("subrounds", ctypes.c_int64),
-        ("solo_subrounds", ctypes.c_int64), ("barriers", ctypes.c_int64),
+        ("levels", ctypes.c_int64), ("phases", ctypes.c_int64),
+        ("solo_phases", ctypes.c_int64), ("barriers", ctypes.c_int64),
         ("scanned", ctypes.c_int64), ("arcs_walked", ctypes.c_int64),
-        ("compactions", ctypes.c_int64), ("kmax", ctypes.c_int32),
+        ("compactions", ctypes.c_int64), ("hub_arcs", ctypes.c_int64), ("kmax", ctypes.c_int32),
         ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
         ("trace_len", ctypes.c_int32), ("kernel_ms", ctypes.c_double),
-        ("reserved", ctypes.c_int64 * 4),
+        ("reserved", ctypes.c_int64 * 3),
     ]
 
 
 @dataclass
 class Stats:
     levels: int
-    subrounds: int
-    solo_subrounds: int
+    phases: int
+    solo_phases: int
     barriers: int
     scanned: int
     arcs_walked: int
     compactions: int
+    hub_arcs: int
     kmax: int
     grid_blocks: int
     block_threads: int
@@ -89,8 +91,9 @@ class Stats:
 
     @classmethod
     def _from(cls, s: _Stats) -> "Stats":
-        return cls(s.levels, s.subrounds, s.solo_subrounds, s.barriers, s.scanned, s.arcs_walked,
-                   s.compactions, s.kmax, s.grid_blocks, s.block_threads, s.kernel_ms, s.trace_len)
+        return cls(s.levels, s.phases, s.solo_phases, s.barriers, s.scanned, s.arcs_walked,
+                   s.compactions, s.hub_arcs, s.kmax, s.grid_blocks, s.block_threads, s.kernel_ms,
+                   s.trace_len)
 
 
 _lib = None
@@ -164,7 +167,7 @@ def _check_csr_tensors(rowptr, colidx):
 
 def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=None,
                     algo: int = ALGO_PERSISTENT, blocks_per_sm: int = 0, solo_arcs: int = 0,
-                    solo_scan: int = 0, trace=None, stats: bool = False):
+                    solo_scan: int = 0, bloom: bool = True, trace=None, stats: bool = False):
     """Core numbers of the graph (rowptr int64[n+1], colidx int32[m] CUDA tensors).
 
     Runs on the current stream of the tensors' device.  Returns an int32 tensor
@@ -181,7 +184,7 @@ def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=
                    workspace.data_ptr() if workspace is not None else None,
                    workspace.numel() * workspace.element_size() if workspace is not None else 0,
                    trace.data_ptr() if trace is not None else None,
-                   trace.shape[0] if trace is not None else 0)
+                   trace.shape[0] if trace is not None else 0, 0 if bloom else 1)
     st = _Stats()
     with torch.cuda.device(dev):
         rc = _load().kcore_decompose_ex(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,

@@ -1,35 +1,43 @@
-// kc_kernels.cuh -- sm_100a kernels of the k-core hot path.
+// kc_kernels.cuh -- sm_100a kernels of the k-core hot path (v3).
 //
-// One call = one persistent cooperative kernel (k_persistent) that runs the
-// whole decomposition as a device-resident state machine:
+// One call = one persistent cooperative kernel (k_persistent), one CTA per SM,
+// running the whole decomposition as a device-resident state machine.  Per
+// level k (Alg. 1's round) there is ONE grid phase:
 //
-//   INIT   deg[v] = rowptr[v+1]-rowptr[v] into core_out, min-degree reduce    (Alg.1 l.1)
-//   SCAN   level k: frontier <- {v alive : deg[v] == k}; fused min{deg > k};   (Alg.2)
-//          optional alive-list compaction (reading R6)
-//   PEEL   sub-round over frontier slots [s,e): for every arc (v,u):          (Alg.3 l.12-24)
-//          if deg[u] > k: old = atomicSub(&deg[u],1);
-//             old == k+1 -> append u (it reached k: next sub-round)
-//             old <= k   -> atomicAdd(&deg[u],1)  (restore, Fig. 6)
-//             else       -> min_next = min(min_next, old-1)   (level skip, reading R5)
-//   level end: k <- max(k+1, min_next)  (Alg.1 l.9 does k+1; reading R5)
+//   LEVEL(k)  every CTA scans its tiles of the alive list (Alg. 2):
+//             deg[v] == k  -> v is in the k-shell: claim it, append it to the
+//                             CTA's LOCAL frontier (shared memory);
+//             deg[v] >  k  -> running min for the level skip, optional
+//                             alive-list compaction;
+//             then drains its local frontier breadth-first with CTA-local
+//             sub-rounds (__syncthreads only) -- the paper's block-local BFS
+//             of Alg. 3.  For every arc (v,u) (Alg. 3 l.19-24):
+//               if deg[u] > k: old = atomicSub(&deg[u],1)
+//                  old == k+1 -> u reached k: claim it, append it to the next
+//                                local frontier
+//                  old <= k   -> atomicAdd(&deg[u],1)  (restore, Fig. 6)
+//                  else       -> min_next = min(min_next, old-1)    (level skip)
+//   HUB       vertices too big for one CTA (> kHub arcs) or overflowing a
+//             local frontier go to a global queue; a HUB phase splits that
+//             queue's ARCS evenly over every warp of the grid, then drains
+//             the resulting local frontiers the same way.
+//   level end k <- max(k+1, min_next)  (Alg. 1 l.9 does k+1; reading R5)
 //
-// Control.  Every CTA keeps an identical copy of the control state (Ctrl) in
-// shared memory.  A phase ends with a grid barrier whose last arriver takes a
-// SNAPSHOT of the three counters (queue tail, compaction length, min) and
-// resets them; every CTA then advances its Ctrl with the same pure function
-// advance(Ctrl, Snap).  No host round-trip, no serial "leader" logic.
-// Phases whose work is tiny (a few thousand arcs, or a short alive list) are
-// marked `solo`: CTA 0 runs them -- and every following tiny phase, across
-// sub-rounds and levels -- alone with __syncthreads instead of grid barriers,
-// then publishes its Ctrl; the other CTAs wait at one barrier.
+// Scan and drain run concurrently in different CTAs, so a vertex can be seen
+// with deg == k by a scan and reached (old == k+1) by a peel in the same
+// level; a claim bit per vertex (atomicOr) makes removal exactly-once
+// (reading R9).
 //
-// Frontier queue: one array order[n] (every vertex is appended exactly once in
-// the whole run, so it cannot overflow -- cf. the paper's per-block buf[i] and
-// ring buffers) plus qarc[n], the exclusive prefix of the
-// appended vertices' degrees.  A packed 64-bit tail (count<<33 | arcs)
-// reserves slots and their arc range with one atomic, so a peel sub-round
-// splits its ARCS evenly over all warps (hubs are shared by many warps; no
-// degree buckets needed).
+// Control: every CTA keeps an identical copy of the control state in shared
+// memory; a phase ends with a grid barrier whose last arriver snapshots and
+// resets the counters, and every CTA applies the same pure advance().  Phases
+// over a short alive list / few arcs run `solo` on CTA 0 with CTA-local sync.
+//
+// Filter: when a CTA has many arcs to walk and the alive list at level start
+// is short, it builds a Bloom filter of that list in shared memory; arcs whose
+// target is definitely not alive (removed at an earlier level) then skip the
+// scattered deg[] read entirely (the read is the throughput limiter, see
+// DESIGN.md "Measured primitives").
 #pragma once
 
 #include "kc_common.cuh"
@@ -37,47 +45,62 @@
 
 namespace kc {
 
-constexpr int kBlock = 512;
+constexpr int kBlock = 1024;
 constexpr int kWarps = kBlock / 32;
 constexpr int kScanItems = 4;
 constexpr int kScanTile = kBlock * kScanItems;
-constexpr int kStageCap = 256;  // per-warp append stage (>= 32 * kUnroll)
-constexpr int kUnroll = 4;      // arcs per lane in flight per peel batch
+constexpr int kLCap = 1024;          // local frontier capacity (entries)
+constexpr int kHub = 8192;           // arcs; bigger vertices go to the global queue
+constexpr int kGStage = 32;          // per-warp global-queue stage
+constexpr int kOStage = 64;          // per-warp order stage
+constexpr int kBloomBits = 1 << 20;  // 128 KB
+constexpr int kBloomWords = kBloomBits / 32;
+constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
+constexpr int kUnroll = 4;
 constexpr int kBatch = 32 * kUnroll;
 constexpr int kTraceFields = 8;
 
-enum : int32_t { PH_INIT = 0, PH_SCAN = 1, PH_PEEL = 2, PH_DONE = 3 };
+enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
-// Control state; replicated in every CTA, advanced by advance().
 struct Ctrl {
     int32_t phase, solo, k, level_min;
     int32_t compact, src_sel, dst_sel, alive_sel;
     int64_t src_len, alive_len;
-    int64_t s, e, as, ae;         // PEEL: slots [s,e), arcs [as,ae)
-    int64_t lvl_cnt0, lvl_arc0;   // queue tail when the level's scan began
-    int64_t st_levels, st_sub, st_solo_sub, st_bar, st_scanned, st_arcs, st_compact;
+    int64_t s, e, as, ae;          // HUB: global-queue slots [s,e), arcs [as,ae)
+    int64_t gq_cnt, gq_arc;        // global queue consumed so far
+    int64_t ord_lvl0;              // order tail when the level began
+    int64_t level;                 // level index (for the Bloom cache)
+    int64_t st_levels, st_phases, st_solo, st_bar, st_scanned, st_compact, st_hubarcs;
     int32_t st_kmax, st_pad;
 };
 
+static_assert(sizeof(Ctrl) % 16 == 0, "Ctrl is copied as int4");
+
 struct Snap {
-    unsigned long long qtail, alive_out;
+    unsigned long long gq;         // packed global-queue tail
+    unsigned long long ord;        // order tail (= removed vertices)
+    unsigned long long alive_out;  // compaction output length
     int32_t min;
     int32_t pad;
 };
 
 struct Params {
     int64_t n;
-    int32_t solo_arcs;  // PEEL phases with <= this many arcs run solo
-    int32_t solo_scan;  // SCAN phases over <= this many entries run solo
+    int32_t solo_arcs;  // HUB phases with <= this many arcs run solo
+    int32_t solo_scan;  // LEVEL phases over <= this many entries run solo
+    int32_t bloom;      // 0 disables the Bloom filter
+    int32_t pad;
 };
 
 struct State {
-    alignas(128) unsigned long long qtail;      // packed (count << 33) | arcs
+    alignas(128) unsigned long long gq_tail;    // packed (count << 33) | arcs
+    alignas(128) unsigned long long ord_tail;   // vertices written to order[]
     alignas(128) unsigned long long alive_out;  // compaction output length
     alignas(128) int32_t min_next;              // atomicMin target
     alignas(128) uint32_t bar_count;            // grid barrier arrivals (monotone)
     alignas(128) uint32_t bar_gen;              // grid barrier generation
     Snap snap[2];                               // counters at barrier gen, by gen & 1
+    alignas(128) unsigned long long arcs_walked;
     alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
     alignas(128) Params prm;
     int64_t *trace;                             // optional [trace_cap][kTraceFields]
@@ -88,24 +111,36 @@ struct State {
 struct KArgs {
     const int64_t *rowptr;
     const int32_t *colidx;
-    int32_t *deg;  // == core_out
-    int32_t *order;
-    int64_t *qarc;
+    int32_t *deg;       // == core_out
+    int32_t *order;     // removal order (all vertices)
+    uint32_t *claimed;  // claim bit per vertex
+    int32_t *gq_v;      // global queue: vertex, row begin, arc prefix
+    int64_t *gq_beg;
+    int64_t *gq_arc;
     int32_t *alive[2];
     State *S;
     int64_t n;
 };
 
 struct Smem {
-    int32_t sv[kWarps][kStageCap];
-    int32_t sd[kWarps][kStageCap];
+    int32_t lv[2][kLCap];
+    int32_t ld[2][kLCap];
+    int64_t lb[2][kLCap];
+    int64_t lpre[kLCap + 1];
+    int32_t lcnt[2];
+    int32_t gv[kWarps][kGStage];
+    int32_t gd[kWarps][kGStage];
+    int64_t gb[kWarps][kGStage];
+    int32_t ov[kWarps][kOStage];
     unsigned long long scan_q[kWarps];
-    uint32_t scan_k[kWarps];
-    unsigned long long tot_q, base_q;
-    unsigned long long tot_k, base_k;
+    unsigned long long tot_q, base_o, base_k;
     int32_t red_min[kWarps];
+    int64_t bloom_level;
+    int32_t bloom_on;
+    int32_t pad;
     Ctrl ctrl;
     Snap snap;
+    uint32_t bloom[kBloomWords];
 };
 
 // ---------------------------------------------------------------- helpers
@@ -130,6 +165,15 @@ __device__ __forceinline__ unsigned long long globaltimer()
     return t;
 }
 
+__device__ __forceinline__ uint32_t bloom_h1(uint32_t v) { return (v * 0x9E3779B1u) >> 12; }
+__device__ __forceinline__ uint32_t bloom_h2(uint32_t v) { return ((v ^ (v >> 15)) * 0x85EBCA6Bu) >> 12; }
+
+__device__ __forceinline__ bool bloom_maybe(const Smem &sm, uint32_t v)
+{
+    const uint32_t a = bloom_h1(v), b = bloom_h2(v);
+    return ((sm.bloom[a >> 5] >> (a & 31)) & (sm.bloom[b >> 5] >> (b & 31)) & 1u) != 0;
+}
+
 // CTA-wide min, then one atomicMin per CTA
 __device__ __forceinline__ void block_min_atomic(Smem &sm, int v, int32_t *target)
 {
@@ -145,243 +189,213 @@ __device__ __forceinline__ void block_min_atomic(Smem &sm, int v, int32_t *targe
     __syncthreads();
 }
 
-// ----------------------------------------------------------- frontier queue
-// Per-warp append stage in shared memory; flushed with ONE packed atomic.
-__device__ __noinline__ void warp_flush(const KArgs &A, Smem &sm, int wib, int &scnt)
-{
-    const int lane = threadIdx.x & 31;
-    if (scnt == 0) return;
-    __syncwarp();
-    int64_t tot = 0;
-    for (int x = lane; x < scnt; x += 32) tot += sm.sd[wib][x];
-    tot = warp_sum64(tot);
-    unsigned long long base = 0;
-    if (lane == 0)
-        base = atomicAdd(&A.S->qtail, ((unsigned long long)scnt << kArcBits) | (unsigned long long)tot);
-    base = __shfl_sync(kFull, base, 0);
-    const int64_t bc = (int64_t)(base >> kArcBits);
-    int64_t carry = (int64_t)(base & kArcMask);
-    for (int x0 = 0; x0 < scnt; x0 += 32) {
-        const int x = x0 + lane;
-        const int64_t d = (x < scnt) ? (int64_t)sm.sd[wib][x] : 0;
-        int64_t incl = d;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            int64_t t = __shfl_up_sync(kFull, incl, o);
-            if (lane >= o) incl += t;
-        }
-        if (x < scnt) {
-            A.order[bc + x] = sm.sv[wib][x];
-            A.qarc[bc + x] = carry + incl - d;
-        }
-        carry += __shfl_sync(kFull, incl, 31);
-    }
-    __syncwarp();
-    scnt = 0;
-}
-
-// Ballot compaction (Fig. 8(c)) of this warp's hits into its stage.
-__device__ __forceinline__ void warp_append(const KArgs &A, Smem &sm, int wib, int &scnt, bool hit,
-                                            int32_t u, int32_t du)
-{
-    const unsigned b = __ballot_sync(kFull, hit);
-    if (b == 0) return;
-    const int c = __popc(b);
-    if (scnt + c > kStageCap) warp_flush(A, sm, wib, scnt);
-    if (hit) {
-        const int pos = scnt + __popc(b & lanemask_lt());
-        sm.sv[wib][pos] = u;
-        sm.sd[wib][pos] = du;
-    }
-    scnt += c;
-    __syncwarp();
-}
-
-// ------------------------------------------------------------------ INIT
-__device__ void phase_init(const KArgs &A, Smem &sm)
-{
-    int lmin = INT_MAX;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < A.n; v += stride) {
-        const int32_t d = (int32_t)(ld_ro_i64(A.rowptr + v + 1) - ld_ro_i64(A.rowptr + v));
-        A.deg[v] = d;
-        lmin = min(lmin, d);
-    }
-    block_min_atomic(sm, lmin, &A.S->min_next);
-}
-
-// ------------------------------------------------------------------ SCAN
-// Block-wide exclusive scan of (packed frontier count|arcs, kept count).
-__device__ __forceinline__ void block_scan2(Smem &sm, unsigned long long q, uint32_t kk,
-                                            unsigned long long &q_ex, uint32_t &k_ex)
+// Block-wide exclusive scan of one u64 per thread; total in sm.tot_q.
+__device__ __forceinline__ unsigned long long block_excl_scan(Smem &sm, unsigned long long q)
 {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     unsigned long long qi = q;
-    uint32_t ki = kk;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
         unsigned long long t = __shfl_up_sync(kFull, qi, o);
-        uint32_t t2 = __shfl_up_sync(kFull, ki, o);
-        if (lane >= o) { qi += t; ki += t2; }
+        if (lane >= o) qi += t;
     }
-    if (lane == 31) { sm.scan_q[wib] = qi; sm.scan_k[wib] = ki; }
+    if (lane == 31) sm.scan_q[wib] = qi;
     __syncthreads();
     if (wib == 0) {
-        unsigned long long wq = lane < kWarps ? sm.scan_q[lane] : 0ULL;
-        uint32_t wk = lane < kWarps ? sm.scan_k[lane] : 0u;
+        const unsigned long long wq = lane < kWarps ? sm.scan_q[lane] : 0ULL;
         unsigned long long iq = wq;
-        uint32_t ik = wk;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             unsigned long long t = __shfl_up_sync(kFull, iq, o);
-            uint32_t t2 = __shfl_up_sync(kFull, ik, o);
-            if (lane >= o) { iq += t; ik += t2; }
+            if (lane >= o) iq += t;
         }
-        if (lane < kWarps) { sm.scan_q[lane] = iq - wq; sm.scan_k[lane] = ik - wk; }
-        if (lane == kWarps - 1) { sm.tot_q = iq; sm.tot_k = ik; }
+        if (lane < kWarps) sm.scan_q[lane] = iq - wq;
+        if (lane == kWarps - 1) sm.tot_q = iq;
     }
     __syncthreads();
-    q_ex = sm.scan_q[wib] + (qi - q);
-    k_ex = sm.scan_k[wib] + (ki - kk);
+    return sm.scan_q[wib] + (qi - q);
 }
 
-__device__ void phase_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
-{
-    const int k = c.k;
-    const int32_t *src = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
-    int32_t *dst = c.compact ? A.alive[c.dst_sel] : nullptr;
-    const int64_t len = c.src_len;
-    const int64_t ntiles = (len + kScanTile - 1) / kScanTile;
-    int lmin = INT_MAX;
-    for (int64_t t = bid; t < ntiles; t += nblk) {
-        int32_t vv[kScanItems], dd[kScanItems], fd[kScanItems];
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) {
-            const int64_t idx = t * kScanTile + (int64_t)j * kBlock + threadIdx.x;
-            vv[j] = -1;
-            if (idx < len) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)idx;
-        }
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_cg_i32(A.deg + vv[j]) : -1;
-        unsigned long long q = 0;
-        uint32_t keep = 0, fmask = 0, kmask = 0;
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) {
-            fd[j] = 0;
-            if (vv[j] < 0) continue;
-            if (dd[j] == k) {
-                fmask |= 1u << j;
-                fd[j] = (int32_t)(ld_ro_i64(A.rowptr + vv[j] + 1) - ld_ro_i64(A.rowptr + vv[j]));
-                q += kCntOne | (unsigned long long)fd[j];
-            } else if (dd[j] > k) {
-                lmin = min(lmin, dd[j]);
-                if (dst) { kmask |= 1u << j; keep++; }
-            }
-        }
-        unsigned long long q_ex;
-        uint32_t k_ex;
-        block_scan2(sm, q, keep, q_ex, k_ex);
-        if (threadIdx.x == 0) {
-            sm.base_q = sm.tot_q ? atomicAdd(&A.S->qtail, sm.tot_q) : 0ULL;
-            sm.base_k = sm.tot_k ? atomicAdd(&A.S->alive_out, sm.tot_k) : 0ULL;
-        }
-        __syncthreads();
-        int64_t slot = (int64_t)((sm.base_q + q_ex) >> kArcBits);
-        int64_t arc = (int64_t)(((sm.base_q & kArcMask) + (q_ex & kArcMask)));
-        int64_t kpos = (int64_t)(sm.base_k + k_ex);
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) {
-            if (fmask & (1u << j)) {
-                A.order[slot] = vv[j];
-                A.qarc[slot] = arc;
-                slot++;
-                arc += fd[j];
-            }
-            if (kmask & (1u << j)) dst[kpos++] = vv[j];
-        }
-    }
-    block_min_atomic(sm, lmin, &A.S->min_next);
-}
-
-// ------------------------------------------------------------------ PEEL
-// Largest slot i in [s,e) with qarc[i] <= a (warp-cooperative 32-ary search).
-__device__ __forceinline__ int64_t find_slot(const int64_t *qarc, int64_t s, int64_t e, int64_t a)
+// ------------------------------------------------------------ warp stages
+// Removal order: every claimed vertex is recorded once (per-warp stage).
+__device__ __noinline__ void order_flush(const KArgs &A, Smem &sm, int wib, int &ocnt)
 {
     const int lane = threadIdx.x & 31;
+    if (ocnt == 0) return;
+    __syncwarp();
+    unsigned long long base = 0;
+    if (lane == 0) base = atomicAdd(&A.S->ord_tail, (unsigned long long)ocnt);
+    base = __shfl_sync(kFull, base, 0);
+    for (int x = lane; x < ocnt; x += 32) A.order[base + x] = sm.ov[wib][x];
+    __syncwarp();
+    ocnt = 0;
+}
+
+// Global queue: one packed atomic reserves slots and their arc range.
+__device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
+{
+    const int lane = threadIdx.x & 31;
+    if (gcnt == 0) return;
+    __syncwarp();
+    const int64_t d = lane < gcnt ? (int64_t)sm.gd[wib][lane] : 0;
+    int64_t incl = d;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        int64_t t = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += t;
+    }
+    const int64_t tot = __shfl_sync(kFull, incl, 31);
+    unsigned long long base = 0;
+    if (lane == 0)
+        base = atomicAdd(&A.S->gq_tail, ((unsigned long long)gcnt << kArcBits) | (unsigned long long)tot);
+    base = __shfl_sync(kFull, base, 0);
+    const int64_t bc = (int64_t)(base >> kArcBits), ba = (int64_t)(base & kArcMask);
+    if (lane < gcnt) {
+        A.gq_v[bc + lane] = sm.gv[wib][lane];
+        A.gq_beg[bc + lane] = sm.gb[wib][lane];
+        A.gq_arc[bc + lane] = ba + incl - d;
+    }
+    __syncwarp();
+    gcnt = 0;
+}
+
+// Route claimed vertices (one per lane where `won`): record order, then send
+// to the local next frontier `nx` if it is small and fits, else to the global
+// queue.  Zero-degree vertices are only recorded.
+__device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool won, int32_t v,
+                                          int32_t dv, int64_t bv, int nx, int &ocnt, int &gcnt)
+{
+    const int lane = threadIdx.x & 31;
+    unsigned b = __ballot_sync(kFull, won);
+    if (b == 0) return;
+    {
+        const int c = __popc(b);
+        if (ocnt + c > kOStage) order_flush(A, sm, wib, ocnt);
+        if (won) sm.ov[wib][ocnt + __popc(b & lanemask_lt())] = v;
+        ocnt += c;
+    }
+    const bool wantl = won && dv > 0 && dv <= kHub;
+    const unsigned bl = __ballot_sync(kFull, wantl);
+    int lbase = 0;
+    if (bl) {
+        if (lane == __ffs(bl) - 1) lbase = atomicAdd(&sm.lcnt[nx], __popc(bl));
+        lbase = __shfl_sync(kFull, lbase, __ffs(bl) - 1);
+    }
+    bool tog = won && dv > 0 && !wantl;
+    if (wantl) {
+        const int pos = lbase + __popc(bl & lanemask_lt());
+        if (pos < kLCap) {
+            sm.lv[nx][pos] = v;
+            sm.ld[nx][pos] = dv;
+            sm.lb[nx][pos] = bv;
+        } else {
+            tog = true;
+        }
+    }
+    const unsigned bg = __ballot_sync(kFull, tog);
+    if (bg) {
+        const int c = __popc(bg);
+        if (gcnt + c > kGStage) gq_flush(A, sm, wib, gcnt);
+        if (tog) {
+            const int pos = gcnt + __popc(bg & lanemask_lt());
+            sm.gv[wib][pos] = v;
+            sm.gd[wib][pos] = dv;
+            sm.gb[wib][pos] = bv;
+        }
+        gcnt += c;
+    }
+    __syncwarp();
+}
+
+__device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
+{
+    const uint32_t bit = 1u << (v & 31);
+    return (atomicOr(A.claimed + (v >> 5), bit) & bit) == 0u;
+}
+
+// --------------------------------------------------------- arc walking
+// Walk arcs [a0,a1) of a frontier whose entries are i = [s,e) with arc
+// prefix P(i) and row begin B(i); the last entry ends at arc ae.  LOCAL=true:
+// entries live in this CTA's shared-memory list `cur`; else in the global
+// queue.  Hits are routed into local list `nx`.
+template <bool LOCAL>
+__device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, const int cur, const int nx,
+                                     int64_t s, int64_t e, int64_t ae, int64_t a0, int64_t a1,
+                                     bool use_bloom, int &lmin, int &ocnt, int &gcnt)
+{
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    // first entry: largest i in [s,e) with P(i) <= a0 (32-ary search)
     int64_t lo = s, hi = e;
-    while (hi - lo > 32) {
-        const int64_t step = (hi - lo + 31) / 32;
+    while (true) {
+        const int64_t step = hi - lo > 32 ? (hi - lo + 31) / 32 : 1;
         const int64_t p = lo + lane * step;
-        const bool ok = (p < hi) && (ld_cg_i64(qarc + p) <= a);
+        bool ok = false;
+        if (p < hi) ok = (LOCAL ? sm.lpre[p] : ld_cg_i64(A.gq_arc + p)) <= a0;
         const unsigned b = __ballot_sync(kFull, ok);
         const int L = 31 - __clz(b);
         lo = lo + L * step;
+        if (step == 1) break;
         hi = min(hi, lo + step);
     }
-    const int64_t p = lo + lane;
-    const bool ok = (p < hi) && (ld_cg_i64(qarc + p) <= a);
-    const unsigned b = __ballot_sync(kFull, ok);
-    return lo + (31 - __clz(b));
-}
-
-// Walk arcs [a0,a1) of the frontier [s,e) (arc range [.,ae)) with one warp.
-__device__ __forceinline__ void peel_range(const KArgs &A, Smem &sm, const int k, int64_t s,
-                                           int64_t e, int64_t ae, int64_t a0, int64_t a1,
-                                           int &scnt, int &lmin)
-{
-    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    int64_t i = find_slot(A.qarc, s, e, a0);
+    int64_t i = lo;
     int64_t a = a0;
     while (a < a1) {
-        // window: slots i .. i+31, one per lane
         const int64_t j = i + lane;
-        int64_t wq = LLONG_MAX, nxt;
-        if (j < e) wq = ld_cg_i64(A.qarc + j);
-        nxt = __shfl_down_sync(kFull, wq, 1);
-        if (lane == 31) nxt = (j + 1 < e) ? ld_cg_i64(A.qarc + j + 1) : ae;
-        if (j + 1 >= e) nxt = ae;
-        int64_t wbeg = 0;
-        if (j < e && nxt > wq && nxt > a && wq < a1) {
-            const int32_t v = ld_cg_i32(A.order + j);
-            wbeg = ld_ro_i64(A.rowptr + v);
+        int64_t wq = LLONG_MAX, wbeg = 0;
+        if (j < e) {
+            wq = LOCAL ? sm.lpre[j] : ld_cg_i64(A.gq_arc + j);
+            wbeg = LOCAL ? sm.lb[cur][j] : ld_cg_i64(A.gq_beg + j);
         }
+        int64_t nxt = __shfl_down_sync(kFull, wq, 1);
+        if (j + 1 >= e) nxt = ae;
+        else if (lane == 31) nxt = LOCAL ? sm.lpre[j + 1] : ld_cg_i64(A.gq_arc + j + 1);
         const int64_t limit = min(a1, __shfl_sync(kFull, nxt, 31));
         while (a < limit) {
             int32_t u[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
                 const int64_t my = a + r * 32 + lane;
-                u[r] = -1;
-                // slot of arc `my`: highest lane whose window start is <= my
                 int pos = 0;
 #pragma unroll
-                for (int bstep = 16; bstep >= 1; bstep >>= 1) {
-                    const int64_t q = __shfl_sync(kFull, wq, pos + bstep);
-                    if (q <= my) pos += bstep;
+                for (int bs = 16; bs >= 1; bs >>= 1) {
+                    const int64_t q = __shfl_sync(kFull, wq, pos + bs);
+                    if (q <= my) pos += bs;
                 }
                 const int64_t beg = __shfl_sync(kFull, wbeg, pos);
                 const int64_t base = __shfl_sync(kFull, wq, pos);
-                if (my < limit) u[r] = ld_stream_i32(A.colidx + beg + (my - base));
+                u[r] = (my < limit) ? ld_stream_i32(A.colidx + beg + (my - base)) : -1;
+            }
+            if (use_bloom) {
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++)
+                    if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
             }
             int32_t d[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) d[r] = u[r] >= 0 ? ld_cg_i32(A.deg + u[r]) : -1;
+            int old[kUnroll];
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
+            bool hit[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
-                bool hit = false;
-                int32_t du = 0;
-                if (d[r] > k) {
-                    const int old = atomicSub(A.deg + u[r], 1);
-                    if (old == k + 1) {
-                        hit = true;
-                        du = (int32_t)(ld_ro_i64(A.rowptr + u[r] + 1) - ld_ro_i64(A.rowptr + u[r]));
-                    } else if (old <= k) {
-                        atomicAdd(A.deg + u[r], 1);
-                    } else {
-                        lmin = min(lmin, old - 1);
-                    }
+                hit[r] = (old[r] == k + 1);
+                if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
+                else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
+            }
+            if (__any_sync(kFull, hit[0] | hit[1] | hit[2] | hit[3])) {
+                bool won[kUnroll];
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++) won[r] = hit[r] && claim(A, u[r]);
+                int64_t b0[kUnroll], b1[kUnroll];
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++) {
+                    b0[r] = won[r] ? ld_ro_i64(A.rowptr + u[r]) : 0;
+                    b1[r] = won[r] ? ld_ro_i64(A.rowptr + u[r] + 1) : 0;
                 }
-                warp_append(A, sm, wib, scnt, hit, u[r], du);
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++)
+                    route_won(A, sm, wib, won[r], u[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, ocnt, gcnt);
             }
             a += kBatch;
         }
@@ -390,7 +404,153 @@ __device__ __forceinline__ void peel_range(const KArgs &A, Smem &sm, const int k
     }
 }
 
-__device__ void phase_peel(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+// Drain this CTA's local frontier (list `cur`) breadth-first with CTA-local
+// sub-rounds.  Returns the number of arcs walked.
+__device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, bool use_bloom,
+                               int &lmin, int &ocnt, int &gcnt)
+{
+    const int wib = threadIdx.x >> 5;
+    int64_t walked = 0;
+    while (true) {
+        __syncthreads();
+        const int L = min(sm.lcnt[cur], kLCap);
+        if (L == 0) break;
+        // arc prefix of the list
+        const int64_t dv = threadIdx.x < L ? (int64_t)sm.ld[cur][threadIdx.x] : 0;
+        const unsigned long long ex = block_excl_scan(sm, (unsigned long long)dv);
+        if (threadIdx.x < L) sm.lpre[threadIdx.x] = (int64_t)ex;
+        const int64_t T = (int64_t)sm.tot_q;
+        const int nx = cur ^ 1;
+        if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; }
+        __syncthreads();
+        int64_t C = (T + kWarps - 1) / kWarps;
+        C = ((C + kBatch - 1) / kBatch) * kBatch;
+        const int64_t a0 = (int64_t)wib * C;
+        if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, lmin, ocnt, gcnt);
+        walked += T;
+        __syncthreads();
+        if (threadIdx.x == 0) sm.lcnt[cur] = 0;
+        cur = nx;
+    }
+    return walked;
+}
+
+// Bloom filter of the alive list at level start (built once per level).
+__device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
+{
+    for (int w = threadIdx.x; w < kBloomWords; w += kBlock) sm.bloom[w] = 0u;
+    __syncthreads();
+    const int32_t *src = A.alive[c.src_sel];
+    for (int64_t i = threadIdx.x; i < c.src_len; i += kBlock) {
+        const uint32_t v = (uint32_t)ld_cg_i32(src + i);
+        const uint32_t h1 = bloom_h1(v), h2 = bloom_h2(v);
+        atomicOr(&sm.bloom[h1 >> 5], 1u << (h1 & 31));
+        atomicOr(&sm.bloom[h2 >> 5], 1u << (h2 & 31));
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) { sm.bloom_level = c.level; sm.bloom_on = 1; }
+    __syncthreads();
+}
+
+// Decide (CTA-uniform) whether walking `arcs` arcs this phase pays for a filter.
+__device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &sm, int64_t arcs)
+{
+    if (!A.S->prm.bloom || c.src_sel < 0 || c.src_len > kBloomMaxA) return false;
+    if (sm.bloom_on && sm.bloom_level == c.level) return true;
+    if (arcs < 4 * c.src_len + 65536) return false;
+    bloom_build(A, c, sm);
+    return true;
+}
+
+// ------------------------------------------------------------------ INIT
+__device__ void phase_init(const KArgs &A, Smem &sm)
+{
+    int lmin = INT_MAX;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (int64_t v = tid; v < A.n; v += stride) {
+        const int32_t d = (int32_t)(ld_ro_i64(A.rowptr + v + 1) - ld_ro_i64(A.rowptr + v));
+        A.deg[v] = d;
+        lmin = min(lmin, d);
+    }
+    for (int64_t w = tid; w < (A.n + 31) / 32; w += stride) A.claimed[w] = 0u;
+    if (threadIdx.x == 0) { sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; }
+    block_min_atomic(sm, lmin, &A.S->min_next);
+}
+
+// ------------------------------------------------------------------ LEVEL
+__device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+{
+    const int k = c.k;
+    const int wib = threadIdx.x >> 5;
+    const int32_t *src = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
+    int32_t *dst = c.compact ? A.alive[c.dst_sel] : nullptr;
+    const int64_t len = c.src_len;
+    const int64_t ntiles = (len + kScanTile - 1) / kScanTile;
+    int lmin = INT_MAX, ocnt = 0, gcnt = 0;
+    if (threadIdx.x == 0) { sm.lcnt[0] = 0; sm.lcnt[1] = 0; }
+    __syncthreads();
+    for (int64_t t = bid; t < ntiles; t += nblk) {
+        int32_t vv[kScanItems], dd[kScanItems];
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) {
+            const int64_t idx = t * kScanTile + (int64_t)j * kBlock + threadIdx.x;
+            vv[j] = -1;
+            if (idx < len) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)idx;
+        }
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_cg_i32(A.deg + vv[j]) : -1;
+        uint32_t keep = 0, kmask = 0;
+        bool won[kScanItems];
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) {
+            won[j] = false;
+            if (vv[j] < 0) continue;
+            if (dd[j] == k) {
+                won[j] = claim(A, vv[j]);
+            } else if (dd[j] > k) {
+                lmin = min(lmin, dd[j]);
+                if (dst) { kmask |= 1u << j; keep++; }
+            }
+        }
+        int64_t b0[kScanItems], b1[kScanItems];
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) {
+            b0[j] = won[j] ? ld_ro_i64(A.rowptr + vv[j]) : 0;
+            b1[j] = won[j] ? ld_ro_i64(A.rowptr + vv[j] + 1) : 0;
+        }
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++)
+            route_won(A, sm, wib, won[j], vv[j], (int32_t)(b1[j] - b0[j]), b0[j], 0, ocnt, gcnt);
+        if (dst) {
+            const unsigned long long ex = block_excl_scan(sm, keep);
+            if (threadIdx.x == 0) sm.base_k = sm.tot_q ? atomicAdd(&A.S->alive_out, sm.tot_q) : 0ULL;
+            __syncthreads();
+            int64_t kpos = (int64_t)(sm.base_k + ex);
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++)
+                if (kmask & (1u << j)) dst[kpos++] = vv[j];
+        }
+    }
+    __syncthreads();
+    // drain the local frontier found by the scan
+    const int L0 = min(sm.lcnt[0], kLCap);
+    int64_t arcs_est = 0;
+    {
+        const int64_t dv = threadIdx.x < L0 ? (int64_t)sm.ld[0][threadIdx.x] : 0;
+        (void)block_excl_scan(sm, (unsigned long long)dv);
+        arcs_est = (int64_t)sm.tot_q;
+    }
+    const bool bl = want_bloom(A, c, sm, arcs_est);
+    const int64_t walked = local_drain(A, sm, k, 0, bl, lmin, ocnt, gcnt);
+    order_flush(A, sm, wib, ocnt);
+    gq_flush(A, sm, wib, gcnt);
+    if (threadIdx.x == 0 && walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+    block_min_atomic(sm, lmin, &A.S->min_next);
+}
+
+// -------------------------------------------------------------------- HUB
+__device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
 {
     const int wib = threadIdx.x >> 5;
     const int64_t gw = (int64_t)bid * kWarps + wib;
@@ -398,71 +558,81 @@ __device__ void phase_peel(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
     const int64_t T = c.ae - c.as;
     int64_t C = (T + W - 1) / W;
     C = ((C + kBatch - 1) / kBatch) * kBatch;
-    int scnt = 0, lmin = INT_MAX;
+    int lmin = INT_MAX, ocnt = 0, gcnt = 0;
+    if (threadIdx.x == 0) { sm.lcnt[0] = 0; sm.lcnt[1] = 0; }
+    __syncthreads();
+    const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
+    const bool bl = want_bloom(A, c, sm, cta_arcs);
     const int64_t a0 = c.as + gw * C;
-    if (a0 < c.ae) peel_range(A, sm, c.k, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), scnt, lmin);
-    warp_flush(A, sm, wib, scnt);
+    if (a0 < c.ae)
+        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, lmin, ocnt, gcnt);
+    int64_t walked = cta_arcs;
+    walked += local_drain(A, sm, c.k, 0, bl, lmin, ocnt, gcnt);
+    order_flush(A, sm, wib, ocnt);
+    gq_flush(A, sm, wib, gcnt);
+    if (threadIdx.x == 0 && walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
 // ---------------------------------------------------------------- control
-// The pure transition function (Alg.1 l.5-9, Alg.3 l.5 and the level skip).
-// Every CTA applies it to identical inputs, so all copies stay identical.
+// The pure transition function (Alg. 1 l.5-9 and the level skip).  Every CTA
+// applies it to identical inputs, so all copies stay identical.
 __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
 {
-    const int64_t cnt = (int64_t)(sn.qtail >> kArcBits), arcs = (int64_t)(sn.qtail & kArcMask);
+    const int64_t gcnt = (int64_t)(sn.gq >> kArcBits), garc = (int64_t)(sn.gq & kArcMask);
+    const int64_t removed = (int64_t)sn.ord;
     c.level_min = min(c.level_min, sn.min);
-    bool level_end = false, peel = false;
-    int64_t ps = 0, pe = 0, pas = 0, pae = 0;
     int next_k = 0;
+    bool new_level = false;
     if (c.phase == PH_INIT) {
         next_k = (c.level_min == INT_MAX) ? 0 : c.level_min;
         c.level_min = INT_MAX;
-    } else if (c.phase == PH_SCAN) {
-        c.st_scanned += c.src_len;
-        if (c.compact) {
-            c.alive_sel = c.dst_sel;
-            c.alive_len = (int64_t)sn.alive_out;
-            c.st_compact++;
+        c.level = -1;
+        new_level = true;
+    } else {
+        c.st_phases++;
+        if (c.solo) c.st_solo++;
+        if (c.phase == PH_LEVEL) {
+            c.st_scanned += c.src_len;
+            if (c.compact) {
+                c.alive_sel = c.dst_sel;
+                c.alive_len = (int64_t)sn.alive_out;
+                c.st_compact++;
+            }
+        } else {
+            c.st_hubarcs += c.ae - c.as;
         }
-        if (arcs > c.lvl_arc0) { peel = true; ps = c.lvl_cnt0; pe = cnt; pas = c.lvl_arc0; pae = arcs; }
-        else level_end = true;
-    } else if (c.phase == PH_PEEL) {
-        c.st_sub++;
-        if (c.solo) c.st_solo_sub++;
-        c.st_arcs += c.ae - c.as;
-        if (cnt > c.e && arcs > c.ae) { peel = true; ps = c.e; pe = cnt; pas = c.ae; pae = arcs; }
-        else level_end = true;
-    }
-    bool scan = (c.phase == PH_INIT);
-    if (level_end) {
-        if (cnt > c.lvl_cnt0) { c.st_levels++; c.st_kmax = c.k; }
-        if (cnt >= p.n) {
+        if (gcnt > c.gq_cnt) {  // hub / overflow vertices pending: HUB phase
+            c.phase = PH_HUB;
+            c.s = c.gq_cnt; c.e = gcnt; c.as = c.gq_arc; c.ae = garc;
+            c.gq_cnt = gcnt; c.gq_arc = garc;
+            c.solo = (c.ae - c.as) <= (int64_t)p.solo_arcs;
+            return;
+        }
+        // level end
+        if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
+        if (removed >= p.n) {
             c.phase = PH_DONE;
             c.solo = 0;
-        } else {
-            next_k = max(c.k + 1, c.level_min);
-            c.level_min = INT_MAX;
-            scan = true;
+            return;
         }
+        next_k = max(c.k + 1, c.level_min);
+        c.level_min = INT_MAX;
+        new_level = true;
     }
-    if (peel) {
-        c.phase = PH_PEEL;
-        c.solo = (pae - pas) <= (int64_t)p.solo_arcs;
-        c.s = ps; c.e = pe; c.as = pas; c.ae = pae;
-    } else if (scan) {
-        const int64_t live = p.n - cnt;
+    if (new_level) {
+        const int64_t live = p.n - removed;
         const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
         const bool compact = c.alive_sel < 0 ? (live * 4 < p.n) : (live * 2 < src_len);
-        c.phase = PH_SCAN;
+        c.phase = PH_LEVEL;
         c.k = next_k;
+        c.level++;
         c.src_sel = c.alive_sel;
         c.src_len = src_len;
         c.compact = compact ? 1 : 0;
         c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
         c.solo = src_len <= (int64_t)p.solo_scan;
-        c.lvl_cnt0 = cnt;
-        c.lvl_arc0 = arcs;
+        c.ord_lvl0 = removed;
     }
 }
 
@@ -470,7 +640,8 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
 __device__ __forceinline__ Snap take_snapshot(State *S)
 {
     Snap sn;
-    sn.qtail = ld_relaxed_u64(&S->qtail);
+    sn.gq = ld_relaxed_u64(&S->gq_tail);
+    sn.ord = ld_relaxed_u64(&S->ord_tail);
     sn.alive_out = ld_relaxed_u64(&S->alive_out);
     sn.min = ld_relaxed_i32(&S->min_next);
     sn.pad = 0;
@@ -489,23 +660,20 @@ __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &s
     r[1] = (int64_t)clock64();
     r[2] = ((int64_t)c.phase << 8) | ((int64_t)c.solo << 4) | grid;  // phase that ENDED
     r[3] = c.k;
-    r[4] = c.phase == PH_SCAN ? c.src_len : (c.e - c.s);
-    r[5] = c.phase == PH_PEEL ? (c.ae - c.as) : 0;
-    r[6] = (int64_t)(sn.qtail >> kArcBits);
-    r[7] = 0;
+    r[4] = c.phase == PH_LEVEL ? c.src_len : (c.e - c.s);
+    r[5] = c.phase == PH_HUB ? (c.ae - c.as) : 0;
+    r[6] = (int64_t)sn.ord;
+    r[7] = (int64_t)(sn.gq >> kArcBits);
     S->trace_n = i + 1;
 }
 
-// Grid barrier; the last arriver snapshots+resets the counters.  Leaves the
-// snapshot in sm.snap (thread 0 only is guaranteed to see it before the final
-// __syncthreads; all threads after).
+// Grid barrier; the last arriver snapshots+resets the counters.
 __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
 {
     __syncthreads();
     if (threadIdx.x == 0) {
         State *S = A.S;
         const uint32_t gen = ld_acquire_u32(&S->bar_gen);
-        __threadfence();
         const uint32_t t = atom_add_release_u32(&S->bar_count, 1u);
         Snap sn;
         if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
@@ -517,7 +685,8 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
             while (ld_acquire_u32(&S->bar_gen) == gen) {
             }
             const Snap *ps = &S->snap[(gen + 1u) & 1u];
-            sn.qtail = ld_relaxed_u64(&ps->qtail);
+            sn.gq = ld_relaxed_u64(&ps->gq);
+            sn.ord = ld_relaxed_u64(&ps->ord);
             sn.alive_out = ld_relaxed_u64(&ps->alive_out);
             sn.min = ld_relaxed_i32(&ps->min);
             sn.pad = 0;
@@ -529,8 +698,8 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
 
 __device__ __forceinline__ void run_phase(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
 {
-    if (c.phase == PH_SCAN) phase_scan(A, c, sm, bid, nblk);
-    else if (c.phase == PH_PEEL) phase_peel(A, c, sm, bid, nblk);
+    if (c.phase == PH_LEVEL) phase_level(A, c, sm, bid, nblk);
+    else if (c.phase == PH_HUB) phase_hub(A, c, sm, bid, nblk);
 }
 
 // CTA 0 alone: run consecutive solo phases with CTA-local synchronisation.
@@ -555,19 +724,22 @@ __device__ void solo_run(const KArgs &A, Smem &sm, const Params &p)
     }
 }
 
-__global__ void __launch_bounds__(kBlock, 2) k_persistent(KArgs A)
+__device__ __forceinline__ void init_ctrl(Ctrl &z)
 {
-    __shared__ Smem sm;
+    z = Ctrl{};
+    z.phase = PH_INIT;
+    z.level_min = INT_MAX;
+    z.alive_sel = -1;
+    z.src_sel = -1;
+}
+
+__global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
+{
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
     State *S = A.S;
     const Params p = S->prm;
-    if (threadIdx.x == 0) {
-        Ctrl z = {};
-        z.phase = PH_INIT;
-        z.level_min = INT_MAX;
-        z.alive_sel = -1;
-        z.src_sel = -1;
-        sm.ctrl = z;
-    }
+    if (threadIdx.x == 0) init_ctrl(sm.ctrl);
     phase_init(A, sm);
     grid_barrier(A, sm);
     if (threadIdx.x == 0) advance(sm.ctrl, sm.snap, p);
@@ -578,11 +750,8 @@ __global__ void __launch_bounds__(kBlock, 2) k_persistent(KArgs A)
             if (blockIdx.x == 0) solo_run(A, sm, p);
             grid_barrier(A, sm);
             if (threadIdx.x == 0) {
-                const Ctrl *pc = &S->pub;
                 Ctrl c;
-                // plain loads are safe: written before CTA 0's release-arrive,
-                // read after this CTA's acquire; bypass L1 with ld.cg
-                const int4 *src = reinterpret_cast<const int4 *>(pc);
+                const int4 *src = reinterpret_cast<const int4 *>(&S->pub);
                 int4 *dst = reinterpret_cast<int4 *>(&c);
 #pragma unroll
                 for (int w = 0; w < (int)(sizeof(Ctrl) / sizeof(int4)); w++) dst[w] = __ldcg(src + w);
@@ -607,10 +776,15 @@ __global__ void __launch_bounds__(kBlock, 2) k_persistent(KArgs A)
 // -------------------------------------------- host-driven ablation kernels
 // (KCORE_ALGO_HOSTLOOP: the paper's Alg. 1 structure -- one launch per phase
 // and a host read-back of the phase after each.  No solo phases.)
-__global__ void __launch_bounds__(kBlock, 2) k_phase(KArgs A)
+__global__ void __launch_bounds__(kBlock, 1) k_phase(KArgs A)
 {
-    __shared__ Smem sm;
-    if (threadIdx.x == 0) sm.ctrl = A.S->pub;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
+    if (threadIdx.x == 0) {
+        sm.ctrl = A.S->pub;
+        sm.bloom_on = 0;
+        sm.bloom_level = -1;
+    }
     __syncthreads();
     const Ctrl c = sm.ctrl;
     if (c.phase == PH_INIT) phase_init(A, sm);
@@ -630,24 +804,24 @@ __global__ void k_leader(KArgs A, int32_t *phase_out)
     *phase_out = c.phase;
 }
 
-__global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan,
+__global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan, int32_t bloom,
                              int64_t *trace, int64_t trace_cap)
 {
     if (threadIdx.x == 0 && blockIdx.x == 0) {
-        S->qtail = 0ULL;
+        S->gq_tail = 0ULL;
+        S->ord_tail = 0ULL;
         S->alive_out = 0ULL;
         S->min_next = INT_MAX;
         S->bar_count = 0u;
         S->bar_gen = 0u;
-        Ctrl z = {};
-        z.phase = PH_INIT;
-        z.level_min = INT_MAX;
-        z.alive_sel = -1;
-        z.src_sel = -1;
+        S->arcs_walked = 0ULL;
+        Ctrl z;
+        init_ctrl(z);
         S->pub = z;
         S->prm.n = n;
         S->prm.solo_arcs = solo_arcs;
         S->prm.solo_scan = solo_scan;
+        S->prm.bloom = bloom;
         S->trace = trace;
         S->trace_cap = trace ? trace_cap : 0;
         S->trace_n = 0ULL;

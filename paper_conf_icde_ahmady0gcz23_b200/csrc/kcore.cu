@@ -42,8 +42,12 @@ int dev_info(DevInfo &out)
         cudaDeviceGetAttribute(&d.major, cudaDevAttrComputeCapabilityMajor, dev);
         cudaDeviceGetAttribute(&d.minor, cudaDevAttrComputeCapabilityMinor, dev);
         if (d.major != 10) return KCORE_EUNSUPPORTED;
+        const int smem = (int)sizeof(Smem);
+        if (cudaFuncSetAttribute(k_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
+            cudaFuncSetAttribute(k_phase, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
+            return KCORE_ECUDA;
         int occ = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_persistent, kBlock, 0) != cudaSuccess)
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_persistent, kBlock, smem) != cudaSuccess)
             return KCORE_ECUDA;
         d.occ = occ;
         d.init = true;
@@ -57,7 +61,9 @@ size_t al(size_t x) { return (x + 255) & ~(size_t)255; }
 struct Carve {
     State *S;
     int32_t *order;
-    int64_t *qarc;
+    uint32_t *claimed;
+    int32_t *gq_v;
+    int64_t *gq_beg, *gq_arc;
     int32_t *alive0, *alive1;
 };
 
@@ -70,9 +76,13 @@ size_t carve(void *base, int64_t n, Carve *c)
         return p;
     };
     Carve t;
+    const size_t nn = (size_t)(n > 0 ? n : 1);
     t.S = (State *)take(sizeof(State));
-    t.order = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
-    t.qarc = (int64_t *)take(sizeof(int64_t) * (size_t)(n + 1));
+    t.order = (int32_t *)take(sizeof(int32_t) * nn);
+    t.claimed = (uint32_t *)take(sizeof(uint32_t) * ((nn + 31) / 32));
+    t.gq_v = (int32_t *)take(sizeof(int32_t) * nn);
+    t.gq_beg = (int64_t *)take(sizeof(int64_t) * nn);
+    t.gq_arc = (int64_t *)take(sizeof(int64_t) * (nn + 1));
     t.alive0 = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
     if (c) *c = t;
@@ -154,6 +164,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     if (algo == KCORE_ALGO_HOSTLOOP) solo = solo_scan = 0;
     int64_t *trace = opt ? opt->trace_out : nullptr;
     const int64_t trace_cap = (opt && opt->trace_out) ? opt->trace_cap : 0;
+    const int bloom = (opt && (opt->flags & KCORE_FLAG_NO_BLOOM)) ? 0 : 1;
+    const size_t smem = sizeof(Smem);
 
     const size_t need = carve(nullptr, n, nullptr);
     void *ws = nullptr;
@@ -175,7 +187,10 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.colidx = colidx;
     A.deg = core_out;
     A.order = cv.order;
-    A.qarc = cv.qarc;
+    A.claimed = cv.claimed;
+    A.gq_v = cv.gq_v;
+    A.gq_beg = cv.gq_beg;
+    A.gq_arc = cv.gq_arc;
     A.alive[0] = cv.alive0;
     A.alive[1] = cv.alive1;
     A.S = cv.S;
@@ -185,19 +200,19 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaEventCreate(&ev0));
         KC_CUDA(cudaEventCreate(&ev1));
     }
-    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, trace, trace_cap);
+    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, trace, trace_cap);
     KC_CUDA(cudaGetLastError());
     if (stats) KC_CUDA(cudaEventRecord(ev0, st));
     if (algo == KCORE_ALGO_PERSISTENT) {
         void *args[] = {&A};
         KC_CUDA(cudaLaunchCooperativeKernel((const void *)k_persistent, dim3(grid), dim3(kBlock), args,
-                                            0, st));
+                                            smem, st));
     } else {
         KC_CUDA(cudaMallocAsync((void **)&d_phase, sizeof(int32_t), st));
         int32_t ph = PH_INIT;
         int guard = 0;
         while (ph != PH_DONE) {
-            k_phase<<<grid, kBlock, 0, st>>>(A);
+            k_phase<<<grid, kBlock, smem, st>>>(A);
             k_leader<<<1, 1, 0, st>>>(A, d_phase);
             KC_CUDA(cudaGetLastError());
             KC_CUDA(cudaMemcpyAsync(&ph, d_phase, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
@@ -216,12 +231,13 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         cudaEventElapsedTime(&ms, ev0, ev1);
         const Ctrl &c = hS.pub;
         stats->levels = c.st_levels;
-        stats->subrounds = c.st_sub;
-        stats->solo_subrounds = c.st_solo_sub;
+        stats->phases = c.st_phases;
+        stats->solo_phases = c.st_solo;
         stats->barriers = c.st_bar;
         stats->scanned = c.st_scanned;
-        stats->arcs_walked = c.st_arcs;
+        stats->arcs_walked = (int64_t)hS.arcs_walked;
         stats->compactions = c.st_compact;
+        stats->hub_arcs = c.st_hubarcs;
         stats->kmax = c.st_kmax;
         stats->grid_blocks = algo == KCORE_ALGO_PERSISTENT ? grid : grid;
         stats->block_threads = kBlock;

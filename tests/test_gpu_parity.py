@@ -39,8 +39,8 @@ def _check(rp, ci, ref=None, **kw):
     return got
 
 
-VARIANTS = [dict(), dict(solo_arcs=-1), dict(blocks_per_sm=1), dict(algo=kc.ALGO_HOSTLOOP),
-            dict(solo_arcs=1 << 30)]
+VARIANTS = [dict(), dict(solo_arcs=-1, solo_scan=-1), dict(bloom=False), dict(algo=kc.ALGO_HOSTLOOP),
+            dict(solo_arcs=1 << 30, solo_scan=1 << 30)]
 
 
 # ------------------------------------------------------------ paper pins
@@ -70,12 +70,12 @@ def test_bowtie_fan_and_star_clamp():
             a, b = 1 + 2 * i, 2 + 2 * i
             e += [(0, a), (0, b), (a, b)]
         rp, ci = kcgen.csr_from_edges(2 * t + 1, e)
-        for kw in VARIANTS[:3]:
+        for kw in VARIANTS:
             _check(rp, ci, np.full(2 * t + 1, 2, np.int32), **kw)
     for L in (10, 1000, 1_000_000):
         rp = np.concatenate([[0, L], L + np.arange(1, L + 1)]).astype(np.int64)
         ci = np.concatenate([np.arange(1, L + 1), np.zeros(L)]).astype(np.int32)
-        for kw in VARIANTS[:3]:
+        for kw in VARIANTS:
             _check(rp, ci, np.ones(L + 1, np.int32), **kw)
 
 

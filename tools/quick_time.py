@@ -22,7 +22,7 @@ for name in names:
             ms.append(st.kernel_ms)
         best = min(ms)
         print(f"{name} {kw} n={n} arcs={m} gen={tg:.2f}s kernel_ms min={best:.3f} med={sorted(ms)[2]:.3f} "
-              f"Medges/s={m/2/best/1e3:.0f} levels={st.levels} sub={st.subrounds} solo={st.solo_subrounds} "
+              f"Medges/s={m/2/best/1e3:.0f} levels={st.levels} phases={st.phases} solo={st.solo_phases} hub_arcs={st.hub_arcs} "
               f"bar={st.barriers} scanned={st.scanned} compact={st.compactions} kmax={st.kmax} grid={st.grid_blocks}",
               flush=True)
     del r, c
