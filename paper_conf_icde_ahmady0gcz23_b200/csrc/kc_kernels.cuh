@@ -52,7 +52,7 @@ constexpr int kScanTile = kBlock * kScanItems;
 constexpr int kLCap = 1024;          // local frontier capacity (entries)
 constexpr int kHub = 8192;           // arcs; bigger vertices go to the global queue
 constexpr int kGStage = 32;          // per-warp global-queue stage
-constexpr int kOStage = 64;          // per-warp order stage
+constexpr int kLArcs = 12288;        // arc budget of one CTA-local sub-round
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -128,10 +128,10 @@ struct Smem {
     int64_t lb[2][kLCap];
     int64_t lpre[kLCap + 1];
     int32_t lcnt[2];
+    int32_t larc[2];
     int32_t gv[kWarps][kGStage];
     int32_t gd[kWarps][kGStage];
     int64_t gb[kWarps][kGStage];
-    int32_t ov[kWarps][kOStage];
     unsigned long long scan_q[kWarps];
     unsigned long long tot_q, base_o, base_k;
     int32_t red_min[kWarps];
@@ -217,20 +217,6 @@ __device__ __forceinline__ unsigned long long block_excl_scan(Smem &sm, unsigned
 }
 
 // ------------------------------------------------------------ warp stages
-// Removal order: every claimed vertex is recorded once (per-warp stage).
-__device__ __noinline__ void order_flush(const KArgs &A, Smem &sm, int wib, int &ocnt)
-{
-    const int lane = threadIdx.x & 31;
-    if (ocnt == 0) return;
-    __syncwarp();
-    unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(&A.S->ord_tail, (unsigned long long)ocnt);
-    base = __shfl_sync(kFull, base, 0);
-    for (int x = lane; x < ocnt; x += 32) A.order[base + x] = sm.ov[wib][x];
-    __syncwarp();
-    ocnt = 0;
-}
-
 // Global queue: one packed atomic reserves slots and their arc range.
 __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
 {
@@ -259,31 +245,46 @@ __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gc
     gcnt = 0;
 }
 
-// Route claimed vertices (one per lane where `won`): record order, then send
-// to the local next frontier `nx` if it is small and fits, else to the global
-// queue.  Zero-degree vertices are only recorded.
+// Route claimed vertices (one per lane where `won`): reserve their slots in
+// the removal order right away (a vertex is claimed only after every vertex
+// whose processing made it reach k was claimed, so claim-time slots form a
+// valid peel order -- the I4 certificate), then send each to the local next
+// frontier `nx` if it is small and fits the sub-round's arc budget, else to
+// the global queue.  Zero-degree vertices are only recorded.
 __device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool won, int32_t v,
-                                          int32_t dv, int64_t bv, int nx, int &ocnt, int &gcnt)
+                                          int32_t dv, int64_t bv, int nx, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
-    unsigned b = __ballot_sync(kFull, won);
+    const unsigned b = __ballot_sync(kFull, won);
     if (b == 0) return;
     {
-        const int c = __popc(b);
-        if (ocnt + c > kOStage) order_flush(A, sm, wib, ocnt);
-        if (won) sm.ov[wib][ocnt + __popc(b & lanemask_lt())] = v;
-        ocnt += c;
+        const int lead = __ffs(b) - 1;
+        unsigned long long base = 0;
+        if (lane == lead) base = atomicAdd(&A.S->ord_tail, (unsigned long long)__popc(b));
+        base = __shfl_sync(kFull, base, lead);
+        if (won) A.order[base + __popc(b & lanemask_lt())] = v;
     }
-    const bool wantl = won && dv > 0 && dv <= kHub;
-    const unsigned bl = __ballot_sync(kFull, wantl);
+    const bool cand = won && dv > 0 && dv <= kHub;
+    const unsigned bc = __ballot_sync(kFull, cand);
+    bool wantl = false;
     int lbase = 0;
-    if (bl) {
-        if (lane == __ffs(bl) - 1) lbase = atomicAdd(&sm.lcnt[nx], __popc(bl));
-        lbase = __shfl_sync(kFull, lbase, __ffs(bl) - 1);
+    if (bc) {
+        int sumd = cand ? dv : 0;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sumd += __shfl_xor_sync(kFull, sumd, o);
+        const int lead = __ffs(bc) - 1;
+        int oa = 0;
+        if (lane == lead) {
+            oa = atomicAdd(&sm.larc[nx], sumd);
+            if (oa + sumd <= kLArcs) lbase = atomicAdd(&sm.lcnt[nx], __popc(bc));
+        }
+        oa = __shfl_sync(kFull, oa, lead);
+        lbase = __shfl_sync(kFull, lbase, lead);
+        wantl = cand && (oa + sumd <= kLArcs);
     }
     bool tog = won && dv > 0 && !wantl;
     if (wantl) {
-        const int pos = lbase + __popc(bl & lanemask_lt());
+        const int pos = lbase + __popc(bc & lanemask_lt());
         if (pos < kLCap) {
             sm.lv[nx][pos] = v;
             sm.ld[nx][pos] = dv;
@@ -321,7 +322,7 @@ __device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
 template <bool LOCAL>
 __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, const int cur, const int nx,
                                      int64_t s, int64_t e, int64_t ae, int64_t a0, int64_t a1,
-                                     bool use_bloom, int &lmin, int &ocnt, int &gcnt)
+                                     bool use_bloom, int &lmin, int &gcnt)
 {
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     // first entry: largest i in [s,e) with P(i) <= a0 (32-ary search)
@@ -395,7 +396,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
                 }
 #pragma unroll
                 for (int r = 0; r < kUnroll; r++)
-                    route_won(A, sm, wib, won[r], u[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, ocnt, gcnt);
+                    route_won(A, sm, wib, won[r], u[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, gcnt);
             }
             a += kBatch;
         }
@@ -407,7 +408,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
 // Drain this CTA's local frontier (list `cur`) breadth-first with CTA-local
 // sub-rounds.  Returns the number of arcs walked.
 __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, bool use_bloom,
-                               int &lmin, int &ocnt, int &gcnt)
+                               int &lmin, int &gcnt)
 {
     const int wib = threadIdx.x >> 5;
     int64_t walked = 0;
@@ -421,15 +422,15 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         if (threadIdx.x < L) sm.lpre[threadIdx.x] = (int64_t)ex;
         const int64_t T = (int64_t)sm.tot_q;
         const int nx = cur ^ 1;
-        if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; }
+        if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; sm.larc[nx] = 0; }
         __syncthreads();
         int64_t C = (T + kWarps - 1) / kWarps;
         C = ((C + kBatch - 1) / kBatch) * kBatch;
         const int64_t a0 = (int64_t)wib * C;
-        if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, lmin, ocnt, gcnt);
+        if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, lmin, gcnt);
         walked += T;
         __syncthreads();
-        if (threadIdx.x == 0) sm.lcnt[cur] = 0;
+        if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
         cur = nx;
     }
     return walked;
@@ -474,7 +475,7 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
         lmin = min(lmin, d);
     }
     for (int64_t w = tid; w < (A.n + 31) / 32; w += stride) A.claimed[w] = 0u;
-    if (threadIdx.x == 0) { sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; }
+    if (threadIdx.x == 0) { sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
@@ -487,8 +488,8 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     int32_t *dst = c.compact ? A.alive[c.dst_sel] : nullptr;
     const int64_t len = c.src_len;
     const int64_t ntiles = (len + kScanTile - 1) / kScanTile;
-    int lmin = INT_MAX, ocnt = 0, gcnt = 0;
-    if (threadIdx.x == 0) { sm.lcnt[0] = 0; sm.lcnt[1] = 0; }
+    int lmin = INT_MAX, gcnt = 0;
+    if (threadIdx.x == 0) { sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
     __syncthreads();
     for (int64_t t = bid; t < ntiles; t += nblk) {
         int32_t vv[kScanItems], dd[kScanItems];
@@ -521,7 +522,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         }
 #pragma unroll
         for (int j = 0; j < kScanItems; j++)
-            route_won(A, sm, wib, won[j], vv[j], (int32_t)(b1[j] - b0[j]), b0[j], 0, ocnt, gcnt);
+            route_won(A, sm, wib, won[j], vv[j], (int32_t)(b1[j] - b0[j]), b0[j], 0, gcnt);
         if (dst) {
             const unsigned long long ex = block_excl_scan(sm, keep);
             if (threadIdx.x == 0) sm.base_k = sm.tot_q ? atomicAdd(&A.S->alive_out, sm.tot_q) : 0ULL;
@@ -542,8 +543,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         arcs_est = (int64_t)sm.tot_q;
     }
     const bool bl = want_bloom(A, c, sm, arcs_est);
-    const int64_t walked = local_drain(A, sm, k, 0, bl, lmin, ocnt, gcnt);
-    order_flush(A, sm, wib, ocnt);
+    const int64_t walked = local_drain(A, sm, k, 0, bl, lmin, gcnt);
     gq_flush(A, sm, wib, gcnt);
     if (threadIdx.x == 0 && walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
     block_min_atomic(sm, lmin, &A.S->min_next);
@@ -558,17 +558,16 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     const int64_t T = c.ae - c.as;
     int64_t C = (T + W - 1) / W;
     C = ((C + kBatch - 1) / kBatch) * kBatch;
-    int lmin = INT_MAX, ocnt = 0, gcnt = 0;
-    if (threadIdx.x == 0) { sm.lcnt[0] = 0; sm.lcnt[1] = 0; }
+    int lmin = INT_MAX, gcnt = 0;
+    if (threadIdx.x == 0) { sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
     const bool bl = want_bloom(A, c, sm, cta_arcs);
     const int64_t a0 = c.as + gw * C;
     if (a0 < c.ae)
-        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, lmin, ocnt, gcnt);
+        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, lmin, gcnt);
     int64_t walked = cta_arcs;
-    walked += local_drain(A, sm, c.k, 0, bl, lmin, ocnt, gcnt);
-    order_flush(A, sm, wib, ocnt);
+    walked += local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
     gq_flush(A, sm, wib, gcnt);
     if (threadIdx.x == 0 && walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
     block_min_atomic(sm, lmin, &A.S->min_next);
@@ -623,7 +622,7 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
     if (new_level) {
         const int64_t live = p.n - removed;
         const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
-        const bool compact = c.alive_sel < 0 ? (live * 4 < p.n) : (live * 2 < src_len);
+        const bool compact = live * 8 < src_len * 7;  // >= 1/8 of the scan source is dead
         c.phase = PH_LEVEL;
         c.k = next_k;
         c.level++;
