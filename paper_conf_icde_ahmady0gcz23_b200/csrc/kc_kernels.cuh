@@ -51,8 +51,9 @@ constexpr int kScanItems = 4;
 constexpr int kScanTile = kBlock * kScanItems;
 constexpr int kLCap = 1024;          // local frontier capacity (entries)
 constexpr int kHub = 8192;           // arcs; bigger vertices go to the global queue
-constexpr int kGStage = 32;          // per-warp global-queue stage
+constexpr int kGStage = 64;          // per-warp global-queue stage
 constexpr int kLArcs = 12288;        // arc budget of one CTA-local sub-round
+constexpr int kLPhaseArcs = 65536;   // arc budget of all local sub-rounds of one phase
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -129,6 +130,12 @@ struct Smem {
     int64_t lpre[kLCap + 1];
     int32_t lcnt[2];
     int32_t larc[2];
+    int32_t lphase;      // local arcs accepted this phase
+    int32_t removed;     // vertices removed by this CTA this phase (order not recorded)
+    int32_t fit;         // scan: local candidates accepted in this tile
+    int32_t pad2;
+    unsigned long long scan_q2[kWarps];
+    unsigned long long tot_q2, base_g, base_w;
     int32_t gv[kWarps][kGStage];
     int32_t gd[kWarps][kGStage];
     int64_t gb[kWarps][kGStage];
@@ -216,6 +223,38 @@ __device__ __forceinline__ unsigned long long block_excl_scan(Smem &sm, unsigned
     return sm.scan_q[wib] + (qi - q);
 }
 
+// Block-wide exclusive scans of two u64 per thread; totals in tot_q / tot_q2.
+__device__ __forceinline__ void block_excl_scan2(Smem &sm, unsigned long long q, unsigned long long r,
+                                                 unsigned long long &qe, unsigned long long &re)
+{
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    unsigned long long qi = q, ri = r;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long t = __shfl_up_sync(kFull, qi, o);
+        const unsigned long long t2 = __shfl_up_sync(kFull, ri, o);
+        if (lane >= o) { qi += t; ri += t2; }
+    }
+    if (lane == 31) { sm.scan_q[wib] = qi; sm.scan_q2[wib] = ri; }
+    __syncthreads();
+    if (wib == 0) {
+        const unsigned long long wq = lane < kWarps ? sm.scan_q[lane] : 0ULL;
+        const unsigned long long wr = lane < kWarps ? sm.scan_q2[lane] : 0ULL;
+        unsigned long long iq = wq, ir = wr;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long t = __shfl_up_sync(kFull, iq, o);
+            const unsigned long long t2 = __shfl_up_sync(kFull, ir, o);
+            if (lane >= o) { iq += t; ir += t2; }
+        }
+        if (lane < kWarps) { sm.scan_q[lane] = iq - wq; sm.scan_q2[lane] = ir - wr; }
+        if (lane == kWarps - 1) { sm.tot_q = iq; sm.tot_q2 = ir; }
+    }
+    __syncthreads();
+    qe = sm.scan_q[wib] + (qi - q);
+    re = sm.scan_q2[wib] + (ri - r);
+}
+
 // ------------------------------------------------------------ warp stages
 // Global queue: one packed atomic reserves slots and their arc range.
 __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
@@ -259,10 +298,14 @@ __device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, boo
     if (b == 0) return;
     {
         const int lead = __ffs(b) - 1;
-        unsigned long long base = 0;
-        if (lane == lead) base = atomicAdd(&A.S->ord_tail, (unsigned long long)__popc(b));
-        base = __shfl_sync(kFull, base, lead);
-        if (won) A.order[base + __popc(b & lanemask_lt())] = v;
+        if (A.order) {  // peel order requested: slots in claim order
+            unsigned long long base = 0;
+            if (lane == lead) base = atomicAdd(&A.S->ord_tail, (unsigned long long)__popc(b));
+            base = __shfl_sync(kFull, base, lead);
+            if (won) A.order[base + __popc(b & lanemask_lt())] = v;
+        } else if (lane == lead) {
+            atomicAdd(&sm.removed, __popc(b));
+        }
     }
     const bool cand = won && dv > 0 && dv <= kHub;
     const unsigned bc = __ballot_sync(kFull, cand);
@@ -274,13 +317,17 @@ __device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, boo
         for (int o = 16; o > 0; o >>= 1) sumd += __shfl_xor_sync(kFull, sumd, o);
         const int lead = __ffs(bc) - 1;
         int oa = 0;
+        int ok = 0;
         if (lane == lead) {
             oa = atomicAdd(&sm.larc[nx], sumd);
-            if (oa + sumd <= kLArcs) lbase = atomicAdd(&sm.lcnt[nx], __popc(bc));
+            if (oa + sumd <= kLArcs) {
+                const int op = atomicAdd(&sm.lphase, sumd);
+                if (op + sumd <= kLPhaseArcs) { ok = 1; lbase = atomicAdd(&sm.lcnt[nx], __popc(bc)); }
+            }
         }
-        oa = __shfl_sync(kFull, oa, lead);
+        ok = __shfl_sync(kFull, ok, lead);
         lbase = __shfl_sync(kFull, lbase, lead);
-        wantl = cand && (oa + sumd <= kLArcs);
+        wantl = cand && ok;
     }
     bool tog = won && dv > 0 && !wantl;
     if (wantl) {
@@ -489,7 +536,10 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     const int64_t len = c.src_len;
     const int64_t ntiles = (len + kScanTile - 1) / kScanTile;
     int lmin = INT_MAX, gcnt = 0;
-    if (threadIdx.x == 0) { sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
+    if (threadIdx.x == 0) {
+        sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
+        sm.lphase = 0; sm.removed = 0; sm.fit = 0;
+    }
     __syncthreads();
     for (int64_t t = bid; t < ntiles; t += nblk) {
         int32_t vv[kScanItems], dd[kScanItems];
@@ -514,24 +564,100 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
                 if (dst) { kmask |= 1u << j; keep++; }
             }
         }
-        int64_t b0[kScanItems], b1[kScanItems];
+        int64_t b0[kScanItems];
+        int32_t du[kScanItems];
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
             b0[j] = won[j] ? ld_ro_i64(A.rowptr + vv[j]) : 0;
-            b1[j] = won[j] ? ld_ro_i64(A.rowptr + vv[j] + 1) : 0;
+            du[j] = won[j] ? (int32_t)(ld_ro_i64(A.rowptr + vv[j] + 1) - b0[j]) : 0;
         }
+        // (1) local candidates: accepted in scan order while the budgets last
+        unsigned long long lc = 0;  // (count << 32) | arcs
+        uint32_t cmask = 0;
 #pragma unroll
         for (int j = 0; j < kScanItems; j++)
-            route_won(A, sm, wib, won[j], vv[j], (int32_t)(b1[j] - b0[j]), b0[j], 0, gcnt);
-        if (dst) {
-            const unsigned long long ex = block_excl_scan(sm, keep);
-            if (threadIdx.x == 0) sm.base_k = sm.tot_q ? atomicAdd(&A.S->alive_out, sm.tot_q) : 0ULL;
-            __syncthreads();
-            int64_t kpos = (int64_t)(sm.base_k + ex);
+            if (won[j] && du[j] > 0 && du[j] <= kHub) { cmask |= 1u << j; lc += (1ULL << 32) | (uint32_t)du[j]; }
+        unsigned long long lce, dummy;
+        block_excl_scan2(sm, lc, 0ULL, lce, dummy);
+        const int cnt0 = sm.lcnt[0], arc0 = sm.larc[0], ph0 = sm.lphase;
+        uint32_t lmask = 0;
+        {
+            int pc = (int)(lce >> 32), pa = (int)(lce & 0xffffffffu);
 #pragma unroll
-            for (int j = 0; j < kScanItems; j++)
-                if (kmask & (1u << j)) dst[kpos++] = vv[j];
+            for (int j = 0; j < kScanItems; j++) {
+                if (!(cmask & (1u << j))) continue;
+                if (cnt0 + pc < kLCap && arc0 + pa + du[j] <= kLArcs && ph0 + pa + du[j] <= kLPhaseArcs) {
+                    lmask |= 1u << j;
+                    sm.lv[0][cnt0 + pc] = vv[j];
+                    sm.ld[0][cnt0 + pc] = du[j];
+                    sm.lb[0][cnt0 + pc] = b0[j];
+                    atomicMax(&sm.fit, pc + 1);
+                }
+                pc++;
+                pa += du[j];
+            }
         }
+        // (2) the rest go to the global queue; order/removed and compaction counts
+        unsigned long long gqv = 0, wk = 0;
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) {
+            if (won[j] && du[j] > 0 && !(lmask & (1u << j))) gqv += kCntOne | (unsigned long long)du[j];
+            if (won[j]) wk += 1ULL << 32;
+        }
+        wk += keep;
+        __syncthreads();
+        unsigned long long gqe, wke;
+        block_excl_scan2(sm, gqv, wk, gqe, wke);
+        if (threadIdx.x == 0) {
+            // accepted local candidates form a prefix: update the list counters
+            const int fit = sm.fit;
+            sm.fit = 0;
+            sm.base_g = sm.tot_q ? atomicAdd(&A.S->gq_tail, sm.tot_q) : 0ULL;
+            const unsigned long long nw = sm.tot_q2 >> 32, nk = sm.tot_q2 & 0xffffffffULL;
+            sm.base_w = (nw && A.order) ? atomicAdd(&A.S->ord_tail, nw) : 0ULL;
+            if (!A.order) sm.removed += (int)nw;
+            sm.base_k = nk ? atomicAdd(&A.S->alive_out, nk) : 0ULL;
+            sm.lcnt[0] = cnt0 + fit;
+        }
+        // arcs accepted locally: the accepted candidates are the first `fit`
+        // in scan order; their arc total is the prefix at `fit`
+        {
+            int pc = (int)(lce >> 32), pa = (int)(lce & 0xffffffffu);
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++) {
+                if (!(cmask & (1u << j))) continue;
+                if (lmask & (1u << j)) {
+                    // the last accepted candidate publishes the accepted arc total
+                    if (cnt0 + pc + 1 <= kLCap) {
+                        const int end_arcs = pa + du[j];
+                        atomicMax(&sm.larc[0], arc0 + end_arcs);
+                        atomicMax(&sm.lphase, ph0 + end_arcs);
+                    }
+                }
+                pc++;
+                pa += du[j];
+            }
+        }
+        __syncthreads();
+        {
+            int64_t gslot = (int64_t)((sm.base_g + gqe) >> kArcBits);
+            int64_t garc = (int64_t)((sm.base_g & kArcMask) + (gqe & kArcMask));
+            int64_t oslot = (int64_t)(sm.base_w + (wke >> 32));
+            int64_t kpos = (int64_t)(sm.base_k + (wke & 0xffffffffULL));
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++) {
+                if (won[j] && du[j] > 0 && !(lmask & (1u << j))) {
+                    A.gq_v[gslot] = vv[j];
+                    A.gq_beg[gslot] = b0[j];
+                    A.gq_arc[gslot] = garc;
+                    gslot++;
+                    garc += du[j];
+                }
+                if (won[j] && A.order) A.order[oslot++] = vv[j];
+                if (kmask & (1u << j)) dst[kpos++] = vv[j];
+            }
+        }
+        __syncthreads();
     }
     __syncthreads();
     // drain the local frontier found by the scan
@@ -545,7 +671,11 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     const bool bl = want_bloom(A, c, sm, arcs_est);
     const int64_t walked = local_drain(A, sm, k, 0, bl, lmin, gcnt);
     gq_flush(A, sm, wib, gcnt);
-    if (threadIdx.x == 0 && walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+        if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
+    }
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
@@ -559,7 +689,10 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     int64_t C = (T + W - 1) / W;
     C = ((C + kBatch - 1) / kBatch) * kBatch;
     int lmin = INT_MAX, gcnt = 0;
-    if (threadIdx.x == 0) { sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
+    if (threadIdx.x == 0) {
+        sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
+        sm.lphase = 0; sm.removed = 0; sm.fit = 0;
+    }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
     const bool bl = want_bloom(A, c, sm, cta_arcs);
@@ -569,7 +702,11 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     int64_t walked = cta_arcs;
     walked += local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
     gq_flush(A, sm, wib, gcnt);
-    if (threadIdx.x == 0 && walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        if (walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+        if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
+    }
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
