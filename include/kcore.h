@@ -88,7 +88,10 @@ typedef struct {
                              /* reported in kcore_stats.trace_len)                      */
     int32_t flags;           /* KCORE_FLAG_* bits                                        */
     int32_t reserved1;
-    int64_t reserved[2];
+    int64_t *trace_cta_out;  /* optional DEVICE int64[trace_cap][grid][4]: per phase and */
+                             /* CTA, globaltimer at {phase start, end of scan or queue  */
+                             /* walk, end of local drain, barrier arrival}              */
+    int64_t reserved[1];
 } kcore_options;
 
 /* Run statistics (filled when a non-NULL pointer is passed; this makes the

@@ -57,7 +57,7 @@ class _Options(ctypes.Structure):
         ("order_out", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
         ("workspace_bytes", ctypes.c_size_t), ("trace_out", ctypes.c_void_p),
         ("trace_cap", ctypes.c_int64), ("flags", ctypes.c_int32), ("reserved1", ctypes.c_int32),
-        ("reserved", ctypes.c_int64 * 2),
+        ("trace_cta_out", ctypes.c_void_p), ("reserved", ctypes.c_int64 * 1),
     ]
 
 
@@ -167,7 +167,8 @@ def _check_csr_tensors(rowptr, colidx):
 
 def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=None,
                     algo: int = ALGO_PERSISTENT, blocks_per_sm: int = 0, solo_arcs: int = 0,
-                    solo_scan: int = 0, bloom: bool = True, trace=None, stats: bool = False):
+                    solo_scan: int = 0, bloom: bool = True, trace=None, trace_cta=None,
+                    stats: bool = False):
     """Core numbers of the graph (rowptr int64[n+1], colidx int32[m] CUDA tensors).
 
     Runs on the current stream of the tensors' device.  Returns an int32 tensor
@@ -184,7 +185,8 @@ def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=
                    workspace.data_ptr() if workspace is not None else None,
                    workspace.numel() * workspace.element_size() if workspace is not None else 0,
                    trace.data_ptr() if trace is not None else None,
-                   trace.shape[0] if trace is not None else 0, 0 if bloom else 1)
+                   trace.shape[0] if trace is not None else 0, 0 if bloom else 1, 0,
+                   trace_cta.data_ptr() if trace_cta is not None else None)
     st = _Stats()
     with torch.cuda.device(dev):
         rc = _load().kcore_decompose_ex(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,

@@ -51,7 +51,7 @@ constexpr int kScanItems = 4;
 constexpr int kScanTile = kBlock * kScanItems;
 constexpr int kLCap = 1024;          // local frontier capacity (entries)
 constexpr int kHub = 8192;           // arcs; bigger vertices go to the global queue
-constexpr int kGStage = 64;          // per-warp global-queue stage
+constexpr int kGStage = 64;          // per-warp global-queue stage (any size; flushed 32 at a time)
 constexpr int kLArcs = 12288;        // arc budget of one CTA-local sub-round
 constexpr int kLPhaseArcs = 65536;   // arc budget of all local sub-rounds of one phase
 constexpr int kBloomBits = 1 << 20;  // 128 KB
@@ -105,6 +105,7 @@ struct State {
     alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
     alignas(128) Params prm;
     int64_t *trace;                             // optional [trace_cap][kTraceFields]
+    int64_t *trace_cta;                         // optional [trace_cap][grid][4]
     int64_t trace_cap;
     unsigned long long trace_n;
 };
@@ -179,6 +180,17 @@ __device__ __forceinline__ bool bloom_maybe(const Smem &sm, uint32_t v)
 {
     const uint32_t a = bloom_h1(v), b = bloom_h2(v);
     return ((sm.bloom[a >> 5] >> (a & 31)) & (sm.bloom[b >> 5] >> (b & 31)) & 1u) != 0;
+}
+
+// Per-CTA timestamps of the current phase (trace mode only): slot 0 phase
+// start, 1 end of scan / queue walk, 2 end of local drain, 3 barrier arrival.
+// Indexed by the number of grid barriers passed (identical in every CTA).
+__device__ __forceinline__ void cta_time(const KArgs &A, const Ctrl &c, int slot)
+{
+    if (threadIdx.x != 0 || c.solo) return;
+    State *S = A.S;
+    if (!S->trace_cta || c.st_bar >= S->trace_cap) return;
+    S->trace_cta[(c.st_bar * gridDim.x + blockIdx.x) * 4 + slot] = (int64_t)globaltimer();
 }
 
 // CTA-wide min, then one atomicMin per CTA
@@ -262,23 +274,30 @@ __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gc
     const int lane = threadIdx.x & 31;
     if (gcnt == 0) return;
     __syncwarp();
-    const int64_t d = lane < gcnt ? (int64_t)sm.gd[wib][lane] : 0;
-    int64_t incl = d;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        int64_t t = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += t;
-    }
-    const int64_t tot = __shfl_sync(kFull, incl, 31);
+    int64_t tot = 0;
+    for (int x = lane; x < gcnt; x += 32) tot += sm.gd[wib][x];
+    tot = warp_sum64(tot);
     unsigned long long base = 0;
     if (lane == 0)
         base = atomicAdd(&A.S->gq_tail, ((unsigned long long)gcnt << kArcBits) | (unsigned long long)tot);
     base = __shfl_sync(kFull, base, 0);
-    const int64_t bc = (int64_t)(base >> kArcBits), ba = (int64_t)(base & kArcMask);
-    if (lane < gcnt) {
-        A.gq_v[bc + lane] = sm.gv[wib][lane];
-        A.gq_beg[bc + lane] = sm.gb[wib][lane];
-        A.gq_arc[bc + lane] = ba + incl - d;
+    const int64_t bc = (int64_t)(base >> kArcBits);
+    int64_t carry = (int64_t)(base & kArcMask);
+    for (int x0 = 0; x0 < gcnt; x0 += 32) {
+        const int x = x0 + lane;
+        const int64_t d = x < gcnt ? (int64_t)sm.gd[wib][x] : 0;
+        int64_t incl = d;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int64_t t = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl += t;
+        }
+        if (x < gcnt) {
+            A.gq_v[bc + x] = sm.gv[wib][x];
+            A.gq_beg[bc + x] = sm.gb[wib][x];
+            A.gq_arc[bc + x] = carry + incl - d;
+        }
+        carry += __shfl_sync(kFull, incl, 31);
     }
     __syncwarp();
     gcnt = 0;
@@ -536,6 +555,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     const int64_t len = c.src_len;
     const int64_t ntiles = (len + kScanTile - 1) / kScanTile;
     int lmin = INT_MAX, gcnt = 0;
+    cta_time(A, c, 0);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
@@ -660,6 +680,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         __syncthreads();
     }
     __syncthreads();
+    cta_time(A, c, 1);
     // drain the local frontier found by the scan
     const int L0 = min(sm.lcnt[0], kLCap);
     int64_t arcs_est = 0;
@@ -670,6 +691,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     }
     const bool bl = want_bloom(A, c, sm, arcs_est);
     const int64_t walked = local_drain(A, sm, k, 0, bl, lmin, gcnt);
+    cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -689,6 +711,7 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     int64_t C = (T + W - 1) / W;
     C = ((C + kBatch - 1) / kBatch) * kBatch;
     int lmin = INT_MAX, gcnt = 0;
+    cta_time(A, c, 0);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
@@ -700,7 +723,10 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     if (a0 < c.ae)
         walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, lmin, gcnt);
     int64_t walked = cta_arcs;
+    __syncthreads();
+    cta_time(A, c, 1);
     walked += local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
+    cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -799,7 +825,7 @@ __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &s
     r[4] = c.phase == PH_LEVEL ? c.src_len : (c.e - c.s);
     r[5] = c.phase == PH_HUB ? (c.ae - c.as) : 0;
     r[6] = (int64_t)sn.ord;
-    r[7] = (int64_t)(sn.gq >> kArcBits);
+    r[7] = c.st_bar;
     S->trace_n = i + 1;
 }
 
@@ -807,6 +833,7 @@ __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &s
 __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
 {
     __syncthreads();
+    cta_time(A, sm.ctrl, 3);
     if (threadIdx.x == 0) {
         State *S = A.S;
         const uint32_t gen = ld_acquire_u32(&S->bar_gen);
@@ -941,7 +968,7 @@ __global__ void k_leader(KArgs A, int32_t *phase_out)
 }
 
 __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan, int32_t bloom,
-                             int64_t *trace, int64_t trace_cap)
+                             int64_t *trace, int64_t *trace_cta, int64_t trace_cap)
 {
     if (threadIdx.x == 0 && blockIdx.x == 0) {
         S->gq_tail = 0ULL;
@@ -959,6 +986,7 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
         S->prm.solo_scan = solo_scan;
         S->prm.bloom = bloom;
         S->trace = trace;
+        S->trace_cta = trace_cta;
         S->trace_cap = trace ? trace_cap : 0;
         S->trace_n = 0ULL;
     }

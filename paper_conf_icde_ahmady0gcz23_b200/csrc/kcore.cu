@@ -200,7 +200,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaEventCreate(&ev0));
         KC_CUDA(cudaEventCreate(&ev1));
     }
-    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, trace, trace_cap);
+    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, trace,
+                                   trace ? opt->trace_cta_out : nullptr, trace_cap);
     KC_CUDA(cudaGetLastError());
     if (stats) KC_CUDA(cudaEventRecord(ev0, st));
     if (algo == KCORE_ALGO_PERSISTENT) {
