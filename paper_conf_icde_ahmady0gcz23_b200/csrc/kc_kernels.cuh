@@ -45,11 +45,11 @@
 
 namespace kc {
 
-constexpr int kBlock = 1024;
+constexpr int kBlock = 768;
 constexpr int kWarps = kBlock / 32;
 constexpr int kScanItems = 4;
 constexpr int kScanTile = kBlock * kScanItems;
-constexpr int kLCap = 1024;          // local frontier capacity (entries)
+constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)
 constexpr int kHub = 8192;           // arcs; bigger vertices go to the global queue
 constexpr int kGStage = 64;          // per-warp global-queue stage (any size; flushed 32 at a time)
 constexpr int kLArcs = 12288;        // arc budget of one CTA-local sub-round
@@ -57,7 +57,7 @@ constexpr int kLPhaseArcs = 65536;   // arc budget of all local sub-rounds of on
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
-constexpr int kUnroll = 4;
+constexpr int kUnroll = 4;  // arcs per lane in flight per batch (handle_hits assumes 4)
 constexpr int kBatch = 32 * kUnroll;
 constexpr int kTraceFields = 8;
 
@@ -381,16 +381,38 @@ __device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
 }
 
 // --------------------------------------------------------- arc walking
+// Hits of one batch (u reached k): claim, fetch row bounds, prefetch the
+// row's first line for the next hop, route.  Out of line: rare path.
+__device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u0, int u1, int u2, int u3,
+                                         unsigned hm, int &gcnt)
+{
+    const int wib = threadIdx.x >> 5;
+    const int uu[4] = {u0, u1, u2, u3};
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        const bool won = ((hm >> r) & 1u) && claim(A, uu[r]);
+        int64_t b0 = 0, b1 = 0;
+        if (won) {
+            b0 = ld_ro_i64(A.rowptr + uu[r]);
+            b1 = ld_ro_i64(A.rowptr + uu[r] + 1);
+            asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0));
+        }
+        route_won(A, sm, wib, won, uu[r], (int32_t)(b1 - b0), b0, nx, gcnt);
+    }
+}
+
 // Walk arcs [a0,a1) of a frontier whose entries are i = [s,e) with arc
 // prefix P(i) and row begin B(i); the last entry ends at arc ae.  LOCAL=true:
 // entries live in this CTA's shared-memory list `cur`; else in the global
-// queue.  Hits are routed into local list `nx`.
+// queue.  Hits are routed into local list `nx`.  Each lane holds one entry
+// of a 32-entry window; an arc finds its entry with a 5-step shuffle search
+// on 32-bit offsets relative to the current batch.
 template <bool LOCAL>
 __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, const int cur, const int nx,
                                      int64_t s, int64_t e, int64_t ae, int64_t a0, int64_t a1,
                                      bool use_bloom, int &lmin, int &gcnt)
 {
-    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int lane = threadIdx.x & 31;
     // first entry: largest i in [s,e) with P(i) <= a0 (32-ary search)
     int64_t lo = s, hi = e;
     while (true) {
@@ -417,20 +439,24 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
         if (j + 1 >= e) nxt = ae;
         else if (lane == 31) nxt = LOCAL ? sm.lpre[j + 1] : ld_cg_i64(A.gq_arc + j + 1);
         const int64_t limit = min(a1, __shfl_sync(kFull, nxt, 31));
+        const int64_t bmq = wbeg - wq;  // colidx index of arc x in this entry = bmq + x
         while (a < limit) {
+            // window starts relative to this batch, clamped to int32
+            const int64_t rq = wq - a;
+            const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
+            const int32_t lim = (int32_t)min((int64_t)kBatch, limit - a);
             int32_t u[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
-                const int64_t my = a + r * 32 + lane;
+                const int32_t my = r * 32 + lane;
                 int pos = 0;
 #pragma unroll
                 for (int bs = 16; bs >= 1; bs >>= 1) {
-                    const int64_t q = __shfl_sync(kFull, wq, pos + bs);
+                    const int32_t q = __shfl_sync(kFull, q32, pos + bs);
                     if (q <= my) pos += bs;
                 }
-                const int64_t beg = __shfl_sync(kFull, wbeg, pos);
-                const int64_t base = __shfl_sync(kFull, wq, pos);
-                u[r] = (my < limit) ? ld_stream_i32(A.colidx + beg + (my - base)) : -1;
+                const int64_t off = __shfl_sync(kFull, bmq, pos);
+                u[r] = (my < lim) ? ld_stream_i32(A.colidx + off + a + my) : -1;
             }
             if (use_bloom) {
 #pragma unroll
@@ -443,27 +469,14 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             int old[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
-            bool hit[kUnroll];
+            unsigned hm = 0;
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
-                hit[r] = (old[r] == k + 1);
-                if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
+                if (old[r] == k + 1) hm |= 1u << r;
+                else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
                 else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
             }
-            if (__any_sync(kFull, hit[0] | hit[1] | hit[2] | hit[3])) {
-                bool won[kUnroll];
-#pragma unroll
-                for (int r = 0; r < kUnroll; r++) won[r] = hit[r] && claim(A, u[r]);
-                int64_t b0[kUnroll], b1[kUnroll];
-#pragma unroll
-                for (int r = 0; r < kUnroll; r++) {
-                    b0[r] = won[r] ? ld_ro_i64(A.rowptr + u[r]) : 0;
-                    b1[r] = won[r] ? ld_ro_i64(A.rowptr + u[r] + 1) : 0;
-                }
-#pragma unroll
-                for (int r = 0; r < kUnroll; r++)
-                    route_won(A, sm, wib, won[r], u[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, gcnt);
-            }
+            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, gcnt);
             a += kBatch;
         }
         a = limit;
