@@ -47,13 +47,12 @@ namespace kc {
 
 constexpr int kBlock = 768;
 constexpr int kWarps = kBlock / 32;
-constexpr int kScanItems = 4;
-constexpr int kScanTile = kBlock * kScanItems;
+constexpr int kScanItems = 8;        // alive-list entries per lane per warp step
 constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)
 constexpr int kHub = 8192;           // arcs; bigger vertices go to the global queue
 constexpr int kGStage = 64;          // per-warp global-queue stage (any size; flushed 32 at a time)
-constexpr int kLArcs = 12288;        // arc budget of one CTA-local sub-round
-constexpr int kLPhaseArcs = 65536;   // arc budget of all local sub-rounds of one phase
+constexpr int kLArcs = 8192;         // arc budget of one CTA-local sub-round
+constexpr int kLPhaseArcs = 16384;   // arc budget of all local sub-rounds of one phase
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -119,7 +118,11 @@ struct KArgs {
     int32_t *gq_v;      // global queue: vertex, row begin, arc prefix
     int64_t *gq_beg;
     int64_t *gq_arc;
-    int32_t *alive[2];
+    int32_t *alive[2];  // alive lists, partitioned into nseg per-CTA segments
+    int32_t *seg_len[2];  // entries of segment b in alive[x]: seg_len[x][b]
+    int64_t seg_R;        // segment region size: segment b lives at [b*R, b*R + len)
+    int32_t nseg;         // = persistent grid size
+    int32_t pad;
     State *S;
     int64_t n;
 };
@@ -133,8 +136,8 @@ struct Smem {
     int32_t larc[2];
     int32_t lphase;      // local arcs accepted this phase
     int32_t removed;     // vertices removed by this CTA this phase (order not recorded)
-    int32_t fit;         // scan: local candidates accepted in this tile
-    int32_t pad2;
+    int32_t fit;         // unused
+    int32_t kcur;        // scan: compaction cursor within the current segment
     unsigned long long scan_q2[kWarps];
     unsigned long long tot_q2, base_g, base_w;
     int32_t gv[kWarps][kGStage];
@@ -520,12 +523,15 @@ __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
 {
     for (int w = threadIdx.x; w < kBloomWords; w += kBlock) sm.bloom[w] = 0u;
     __syncthreads();
-    const int32_t *src = A.alive[c.src_sel];
-    for (int64_t i = threadIdx.x; i < c.src_len; i += kBlock) {
-        const uint32_t v = (uint32_t)ld_cg_i32(src + i);
-        const uint32_t h1 = bloom_h1(v), h2 = bloom_h2(v);
-        atomicOr(&sm.bloom[h1 >> 5], 1u << (h1 & 31));
-        atomicOr(&sm.bloom[h2 >> 5], 1u << (h2 & 31));
+    for (int b = 0; b < A.nseg; b++) {
+        const int32_t *src = A.alive[c.src_sel] + (int64_t)b * A.seg_R;
+        const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
+        for (int64_t i = threadIdx.x; i < len; i += kBlock) {
+            const uint32_t v = (uint32_t)ld_cg_i32(src + i);
+            const uint32_t h1 = bloom_h1(v), h2 = bloom_h2(v);
+            atomicOr(&sm.bloom[h1 >> 5], 1u << (h1 & 31));
+            atomicOr(&sm.bloom[h2 >> 5], 1u << (h2 & 31));
+        }
     }
     __syncthreads();
     if (threadIdx.x == 0) { sm.bloom_level = c.level; sm.bloom_on = 1; }
@@ -559,14 +565,79 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
 }
 
 // ------------------------------------------------------------------ LEVEL
-__device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+// Scan one alive-list segment (Alg. 2): warps walk it independently, eight
+// entries per lane in flight; deg == k -> claim + route (local frontier or
+// global queue); deg > k -> min for the level skip and, when compacting,
+// ballot-compaction (Fig. 8(c)) into the same segment of the other buffer.
+// No block-wide synchronisation and no global atomics per tile.
+__device__ void scan_segment(const KArgs &A, const Ctrl &c, Smem &sm, int seg, int &lmin, int &gcnt)
 {
     const int k = c.k;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int64_t base = (int64_t)seg * A.seg_R;
+    int64_t len;
+    if (c.src_sel < 0) len = max((int64_t)0, min(A.seg_R, A.n - base));
+    else len = ld_cg_i32(A.seg_len[c.src_sel] + seg);
+    const int32_t *src = c.src_sel < 0 ? nullptr : A.alive[c.src_sel] + base;
+    int32_t *dst = c.compact ? A.alive[c.dst_sel] + base : nullptr;
+    if (threadIdx.x == 0) sm.kcur = 0;
+    __syncthreads();
+    constexpr int CH = 32 * kScanItems;
+    for (int64_t off = (int64_t)wib * CH; off < len; off += (int64_t)kWarps * CH) {
+        int32_t vv[kScanItems], dd[kScanItems];
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) {
+            const int64_t idx = off + j * 32 + lane;
+            vv[j] = -1;
+            if (idx < len) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)(base + idx);
+        }
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_cg_i32(A.deg + vv[j]) : -1;
+        bool won[kScanItems];
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) {
+            won[j] = false;
+            if (dd[j] == k) won[j] = claim(A, vv[j]);
+            else if (dd[j] > k) lmin = min(lmin, dd[j]);
+        }
+        if (dst) {
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++) {
+                const bool keep = dd[j] > k;
+                const unsigned b = __ballot_sync(kFull, keep);
+                if (b) {
+                    int pos = 0;
+                    if (lane == 0) pos = atomicAdd(&sm.kcur, __popc(b));
+                    pos = __shfl_sync(kFull, pos, 0);
+                    if (keep) dst[pos + __popc(b & lanemask_lt())] = vv[j];
+                }
+            }
+        }
+        if (__any_sync(kFull, won[0] | won[1] | won[2] | won[3] | won[4] | won[5] | won[6] | won[7])) {
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++) {
+                int64_t b0 = 0, b1 = 0;
+                if (won[j]) {
+                    b0 = ld_ro_i64(A.rowptr + vv[j]);
+                    b1 = ld_ro_i64(A.rowptr + vv[j] + 1);
+                    asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0));
+                }
+                route_won(A, sm, wib, won[j], vv[j], (int32_t)(b1 - b0), b0, 0, gcnt);
+            }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && dst) {
+        A.seg_len[c.dst_sel][seg] = sm.kcur;
+        if (sm.kcur) atomicAdd(&A.S->alive_out, (unsigned long long)sm.kcur);
+    }
+}
+
+// One level (Alg. 1 round k): scan this CTA's segment(s), then drain the
+// local frontier breadth-first.
+__device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+{
     const int wib = threadIdx.x >> 5;
-    const int32_t *src = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
-    int32_t *dst = c.compact ? A.alive[c.dst_sel] : nullptr;
-    const int64_t len = c.src_len;
-    const int64_t ntiles = (len + kScanTile - 1) / kScanTile;
     int lmin = INT_MAX, gcnt = 0;
     cta_time(A, c, 0);
     if (threadIdx.x == 0) {
@@ -574,136 +645,15 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
     }
     __syncthreads();
-    for (int64_t t = bid; t < ntiles; t += nblk) {
-        int32_t vv[kScanItems], dd[kScanItems];
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) {
-            const int64_t idx = t * kScanTile + (int64_t)j * kBlock + threadIdx.x;
-            vv[j] = -1;
-            if (idx < len) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)idx;
-        }
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_cg_i32(A.deg + vv[j]) : -1;
-        uint32_t keep = 0, kmask = 0;
-        bool won[kScanItems];
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) {
-            won[j] = false;
-            if (vv[j] < 0) continue;
-            if (dd[j] == k) {
-                won[j] = claim(A, vv[j]);
-            } else if (dd[j] > k) {
-                lmin = min(lmin, dd[j]);
-                if (dst) { kmask |= 1u << j; keep++; }
-            }
-        }
-        int64_t b0[kScanItems];
-        int32_t du[kScanItems];
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) {
-            b0[j] = won[j] ? ld_ro_i64(A.rowptr + vv[j]) : 0;
-            du[j] = won[j] ? (int32_t)(ld_ro_i64(A.rowptr + vv[j] + 1) - b0[j]) : 0;
-        }
-        // (1) local candidates: accepted in scan order while the budgets last
-        unsigned long long lc = 0;  // (count << 32) | arcs
-        uint32_t cmask = 0;
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++)
-            if (won[j] && du[j] > 0 && du[j] <= kHub) { cmask |= 1u << j; lc += (1ULL << 32) | (uint32_t)du[j]; }
-        unsigned long long lce, dummy;
-        block_excl_scan2(sm, lc, 0ULL, lce, dummy);
-        const int cnt0 = sm.lcnt[0], arc0 = sm.larc[0], ph0 = sm.lphase;
-        uint32_t lmask = 0;
-        {
-            int pc = (int)(lce >> 32), pa = (int)(lce & 0xffffffffu);
-#pragma unroll
-            for (int j = 0; j < kScanItems; j++) {
-                if (!(cmask & (1u << j))) continue;
-                if (cnt0 + pc < kLCap && arc0 + pa + du[j] <= kLArcs && ph0 + pa + du[j] <= kLPhaseArcs) {
-                    lmask |= 1u << j;
-                    sm.lv[0][cnt0 + pc] = vv[j];
-                    sm.ld[0][cnt0 + pc] = du[j];
-                    sm.lb[0][cnt0 + pc] = b0[j];
-                    atomicMax(&sm.fit, pc + 1);
-                }
-                pc++;
-                pa += du[j];
-            }
-        }
-        // (2) the rest go to the global queue; order/removed and compaction counts
-        unsigned long long gqv = 0, wk = 0;
-#pragma unroll
-        for (int j = 0; j < kScanItems; j++) {
-            if (won[j] && du[j] > 0 && !(lmask & (1u << j))) gqv += kCntOne | (unsigned long long)du[j];
-            if (won[j]) wk += 1ULL << 32;
-        }
-        wk += keep;
-        __syncthreads();
-        unsigned long long gqe, wke;
-        block_excl_scan2(sm, gqv, wk, gqe, wke);
-        if (threadIdx.x == 0) {
-            // accepted local candidates form a prefix: update the list counters
-            const int fit = sm.fit;
-            sm.fit = 0;
-            sm.base_g = sm.tot_q ? atomicAdd(&A.S->gq_tail, sm.tot_q) : 0ULL;
-            const unsigned long long nw = sm.tot_q2 >> 32, nk = sm.tot_q2 & 0xffffffffULL;
-            sm.base_w = (nw && A.order) ? atomicAdd(&A.S->ord_tail, nw) : 0ULL;
-            if (!A.order) sm.removed += (int)nw;
-            sm.base_k = nk ? atomicAdd(&A.S->alive_out, nk) : 0ULL;
-            sm.lcnt[0] = cnt0 + fit;
-        }
-        // arcs accepted locally: the accepted candidates are the first `fit`
-        // in scan order; their arc total is the prefix at `fit`
-        {
-            int pc = (int)(lce >> 32), pa = (int)(lce & 0xffffffffu);
-#pragma unroll
-            for (int j = 0; j < kScanItems; j++) {
-                if (!(cmask & (1u << j))) continue;
-                if (lmask & (1u << j)) {
-                    // the last accepted candidate publishes the accepted arc total
-                    if (cnt0 + pc + 1 <= kLCap) {
-                        const int end_arcs = pa + du[j];
-                        atomicMax(&sm.larc[0], arc0 + end_arcs);
-                        atomicMax(&sm.lphase, ph0 + end_arcs);
-                    }
-                }
-                pc++;
-                pa += du[j];
-            }
-        }
-        __syncthreads();
-        {
-            int64_t gslot = (int64_t)((sm.base_g + gqe) >> kArcBits);
-            int64_t garc = (int64_t)((sm.base_g & kArcMask) + (gqe & kArcMask));
-            int64_t oslot = (int64_t)(sm.base_w + (wke >> 32));
-            int64_t kpos = (int64_t)(sm.base_k + (wke & 0xffffffffULL));
-#pragma unroll
-            for (int j = 0; j < kScanItems; j++) {
-                if (won[j] && du[j] > 0 && !(lmask & (1u << j))) {
-                    A.gq_v[gslot] = vv[j];
-                    A.gq_beg[gslot] = b0[j];
-                    A.gq_arc[gslot] = garc;
-                    gslot++;
-                    garc += du[j];
-                }
-                if (won[j] && A.order) A.order[oslot++] = vv[j];
-                if (kmask & (1u << j)) dst[kpos++] = vv[j];
-            }
-        }
-        __syncthreads();
+    if (nblk == 1) {
+        for (int seg = 0; seg < A.nseg; seg++) scan_segment(A, c, sm, seg, lmin, gcnt);
+    } else {
+        scan_segment(A, c, sm, bid, lmin, gcnt);
     }
     __syncthreads();
     cta_time(A, c, 1);
-    // drain the local frontier found by the scan
-    const int L0 = min(sm.lcnt[0], kLCap);
-    int64_t arcs_est = 0;
-    {
-        const int64_t dv = threadIdx.x < L0 ? (int64_t)sm.ld[0][threadIdx.x] : 0;
-        (void)block_excl_scan(sm, (unsigned long long)dv);
-        arcs_est = (int64_t)sm.tot_q;
-    }
-    const bool bl = want_bloom(A, c, sm, arcs_est);
-    const int64_t walked = local_drain(A, sm, k, 0, bl, lmin, gcnt);
+    const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
+    const int64_t walked = local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();

@@ -65,7 +65,10 @@ struct Carve {
     int32_t *gq_v;
     int64_t *gq_beg, *gq_arc;
     int32_t *alive0, *alive1;
+    int32_t *seg0, *seg1;
 };
+
+constexpr int kMaxSeg = 4096;  // persistent grids are far smaller (148 x occupancy)
 
 size_t carve(void *base, int64_t n, Carve *c)
 {
@@ -83,8 +86,10 @@ size_t carve(void *base, int64_t n, Carve *c)
     t.gq_v = (int32_t *)take(sizeof(int32_t) * nn);
     t.gq_beg = (int64_t *)take(sizeof(int64_t) * nn);
     t.gq_arc = (int64_t *)take(sizeof(int64_t) * (nn + 1));
-    t.alive0 = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
-    t.alive1 = (int32_t *)take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    t.alive0 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
+    t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
+    t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
+    t.seg1 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     if (c) *c = t;
     return off;
 }
@@ -156,6 +161,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     if (bps > di.occ) bps = di.occ;
     if (bps < 1) return KCORE_EUNSUPPORTED;
     const int grid = di.sms * bps;
+    if (grid > kMaxSeg) return KCORE_EUNSUPPORTED;
     int solo = default_solo_arcs(), solo_scan = default_solo_scan();
     if (opt && opt->solo_arcs > 0) solo = opt->solo_arcs;
     if (opt && opt->solo_arcs < 0) solo = 0;
@@ -193,6 +199,11 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.gq_arc = cv.gq_arc;
     A.alive[0] = cv.alive0;
     A.alive[1] = cv.alive1;
+    A.seg_len[0] = cv.seg0;
+    A.seg_len[1] = cv.seg1;
+    A.nseg = grid;
+    A.seg_R = (n + grid - 1) / grid;
+    A.pad = 0;
     A.S = cv.S;
     A.n = n;
 
