@@ -391,16 +391,19 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u
 {
     const int wib = threadIdx.x >> 5;
     const int uu[4] = {u0, u1, u2, u3};
+    bool won[4];
+#pragma unroll
+    for (int r = 0; r < 4; r++) won[r] = ((hm >> r) & 1u) && claim(A, uu[r]);
+    int64_t b0[4], b1[4];
 #pragma unroll
     for (int r = 0; r < 4; r++) {
-        const bool won = ((hm >> r) & 1u) && claim(A, uu[r]);
-        int64_t b0 = 0, b1 = 0;
-        if (won) {
-            b0 = ld_ro_i64(A.rowptr + uu[r]);
-            b1 = ld_ro_i64(A.rowptr + uu[r] + 1);
-            asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0));
-        }
-        route_won(A, sm, wib, won, uu[r], (int32_t)(b1 - b0), b0, nx, gcnt);
+        b0[r] = won[r] ? ld_ro_i64(A.rowptr + uu[r]) : 0;
+        b1[r] = won[r] ? ld_ro_i64(A.rowptr + uu[r] + 1) : 0;
+    }
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        if (won[r] && b1[r] > b0[r]) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[r]));
+        route_won(A, sm, wib, won[r], uu[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, gcnt);
     }
 }
 
@@ -565,11 +568,12 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
 }
 
 // ------------------------------------------------------------------ LEVEL
-// Scan one alive-list segment (Alg. 2): warps walk it independently, eight
-// entries per lane in flight; deg == k -> claim + route (local frontier or
-// global queue); deg > k -> min for the level skip and, when compacting,
-// ballot-compaction (Fig. 8(c)) into the same segment of the other buffer.
-// No block-wide synchronisation and no global atomics per tile.
+// Scan one alive-list segment with ONE warp (Alg. 2): eight entries per lane
+// in flight; deg == k -> claim + route (local frontier or global queue);
+// deg > k -> min for the level skip and, when compacting, ballot compaction
+// (Fig. 8(c)) into the same segment of the other buffer.  Every warp owns a
+// segment for the whole run, so the compaction cursor is a register: no
+// block-wide synchronisation and no global atomics while scanning.
 __device__ void scan_segment(const KArgs &A, const Ctrl &c, Smem &sm, int seg, int &lmin, int &gcnt)
 {
     const int k = c.k;
@@ -580,10 +584,9 @@ __device__ void scan_segment(const KArgs &A, const Ctrl &c, Smem &sm, int seg, i
     else len = ld_cg_i32(A.seg_len[c.src_sel] + seg);
     const int32_t *src = c.src_sel < 0 ? nullptr : A.alive[c.src_sel] + base;
     int32_t *dst = c.compact ? A.alive[c.dst_sel] + base : nullptr;
-    if (threadIdx.x == 0) sm.kcur = 0;
-    __syncthreads();
+    int kcur = 0;
     constexpr int CH = 32 * kScanItems;
-    for (int64_t off = (int64_t)wib * CH; off < len; off += (int64_t)kWarps * CH) {
+    for (int64_t off = 0; off < len; off += CH) {
         int32_t vv[kScanItems], dd[kScanItems];
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
@@ -593,11 +596,10 @@ __device__ void scan_segment(const KArgs &A, const Ctrl &c, Smem &sm, int seg, i
         }
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_cg_i32(A.deg + vv[j]) : -1;
-        bool won[kScanItems];
+        unsigned wm = 0;
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
-            won[j] = false;
-            if (dd[j] == k) won[j] = claim(A, vv[j]);
+            if (dd[j] == k) { if (claim(A, vv[j])) wm |= 1u << j; }
             else if (dd[j] > k) lmin = min(lmin, dd[j]);
         }
         if (dst) {
@@ -605,31 +607,32 @@ __device__ void scan_segment(const KArgs &A, const Ctrl &c, Smem &sm, int seg, i
             for (int j = 0; j < kScanItems; j++) {
                 const bool keep = dd[j] > k;
                 const unsigned b = __ballot_sync(kFull, keep);
-                if (b) {
-                    int pos = 0;
-                    if (lane == 0) pos = atomicAdd(&sm.kcur, __popc(b));
-                    pos = __shfl_sync(kFull, pos, 0);
-                    if (keep) dst[pos + __popc(b & lanemask_lt())] = vv[j];
-                }
+                if (keep) dst[kcur + __popc(b & lanemask_lt())] = vv[j];
+                kcur += __popc(b);
             }
         }
-        if (__any_sync(kFull, won[0] | won[1] | won[2] | won[3] | won[4] | won[5] | won[6] | won[7])) {
+        if (__any_sync(kFull, wm != 0)) {
+            // row bounds of every claimed vertex first (all loads in flight), then route
+            int64_t b0[kScanItems];
+            int32_t du[kScanItems];
 #pragma unroll
             for (int j = 0; j < kScanItems; j++) {
-                int64_t b0 = 0, b1 = 0;
-                if (won[j]) {
-                    b0 = ld_ro_i64(A.rowptr + vv[j]);
-                    b1 = ld_ro_i64(A.rowptr + vv[j] + 1);
-                    asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0));
+                b0[j] = 0; du[j] = 0;
+                if (((wm >> j) & 1u) && k > 0) {  // at k = 0 every claimed vertex is isolated
+                    b0[j] = ld_ro_i64(A.rowptr + vv[j]);
+                    du[j] = (int32_t)(ld_ro_i64(A.rowptr + vv[j] + 1) - b0[j]);
                 }
-                route_won(A, sm, wib, won[j], vv[j], (int32_t)(b1 - b0), b0, 0, gcnt);
+            }
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++) {
+                if (du[j] > 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[j]));
+                route_won(A, sm, wib, (wm >> j) & 1u, vv[j], du[j], b0[j], 0, gcnt);
             }
         }
     }
-    __syncthreads();
-    if (threadIdx.x == 0 && dst) {
-        A.seg_len[c.dst_sel][seg] = sm.kcur;
-        if (sm.kcur) atomicAdd(&A.S->alive_out, (unsigned long long)sm.kcur);
+    if (lane == 0 && dst) {
+        A.seg_len[c.dst_sel][seg] = kcur;
+        if (kcur) atomicAdd(&A.S->alive_out, (unsigned long long)kcur);
     }
 }
 
@@ -645,11 +648,9 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
     }
     __syncthreads();
-    if (nblk == 1) {
-        for (int seg = 0; seg < A.nseg; seg++) scan_segment(A, c, sm, seg, lmin, gcnt);
-    } else {
-        scan_segment(A, c, sm, bid, lmin, gcnt);
-    }
+    // warp w of CTA b owns segment b*kWarps + w; a solo CTA takes all of them
+    for (int seg = bid * kWarps + wib; seg < A.nseg; seg += nblk * kWarps)
+        scan_segment(A, c, sm, seg, lmin, gcnt);
     __syncthreads();
     cta_time(A, c, 1);
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);

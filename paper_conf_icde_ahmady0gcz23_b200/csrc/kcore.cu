@@ -68,7 +68,7 @@ struct Carve {
     int32_t *seg0, *seg1;
 };
 
-constexpr int kMaxSeg = 4096;  // persistent grids are far smaller (148 x occupancy)
+constexpr int kMaxSeg = 16384;  // one alive-list segment per warp of the persistent grid
 
 size_t carve(void *base, int64_t n, Carve *c)
 {
@@ -161,7 +161,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     if (bps > di.occ) bps = di.occ;
     if (bps < 1) return KCORE_EUNSUPPORTED;
     const int grid = di.sms * bps;
-    if (grid > kMaxSeg) return KCORE_EUNSUPPORTED;
+    if (grid * kWarps > kMaxSeg) return KCORE_EUNSUPPORTED;
     int solo = default_solo_arcs(), solo_scan = default_solo_scan();
     if (opt && opt->solo_arcs > 0) solo = opt->solo_arcs;
     if (opt && opt->solo_arcs < 0) solo = 0;
@@ -201,8 +201,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.alive[1] = cv.alive1;
     A.seg_len[0] = cv.seg0;
     A.seg_len[1] = cv.seg1;
-    A.nseg = grid;
-    A.seg_R = (n + grid - 1) / grid;
+    A.nseg = grid * kWarps;
+    A.seg_R = (n + A.nseg - 1) / A.nseg;
     A.pad = 0;
     A.S = cv.S;
     A.n = n;
