@@ -65,6 +65,8 @@ enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 struct Ctrl {
     int32_t phase, solo, k, level_min;
     int32_t compact, src_sel, dst_sel, alive_sel;
+    int32_t src_single, alive_single;  // 1: the list is one contiguous run in segment 0
+    int32_t pad0, pad1;
     int64_t src_len, alive_len;
     int64_t s, e, as, ae;          // HUB: global-queue slots [s,e), arcs [as,ae)
     int64_t gq_cnt, gq_arc;        // global queue consumed so far
@@ -526,15 +528,19 @@ __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
 {
     for (int w = threadIdx.x; w < kBloomWords; w += kBlock) sm.bloom[w] = 0u;
     __syncthreads();
-    for (int b = 0; b < A.nseg; b++) {
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int nseg = c.src_single ? 1 : A.nseg;
+    for (int b = wib; b < nseg; b += kWarps) {  // one warp per segment
         const int32_t *src = A.alive[c.src_sel] + (int64_t)b * A.seg_R;
-        const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
-        for (int64_t i = threadIdx.x; i < len; i += kBlock) {
+        const int64_t len = c.src_single ? c.src_len : ld_cg_i32(A.seg_len[c.src_sel] + b);
+        const int64_t step = c.src_single ? (int64_t)kBlock : 32;
+        for (int64_t i = c.src_single ? threadIdx.x : lane; i < len; i += step) {
             const uint32_t v = (uint32_t)ld_cg_i32(src + i);
             const uint32_t h1 = bloom_h1(v), h2 = bloom_h2(v);
             atomicOr(&sm.bloom[h1 >> 5], 1u << (h1 & 31));
             atomicOr(&sm.bloom[h2 >> 5], 1u << (h2 & 31));
         }
+        if (c.src_single) break;
     }
     __syncthreads();
     if (threadIdx.x == 0) { sm.bloom_level = c.level; sm.bloom_on = 1; }
@@ -568,48 +574,47 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
 }
 
 // ------------------------------------------------------------------ LEVEL
-// Scan one alive-list segment with ONE warp (Alg. 2): eight entries per lane
-// in flight; deg == k -> claim + route (local frontier or global queue);
-// deg > k -> min for the level skip and, when compacting, ballot compaction
-// (Fig. 8(c)) into the same segment of the other buffer.  Every warp owns a
-// segment for the whole run, so the compaction cursor is a register: no
-// block-wide synchronisation and no global atomics while scanning.
-__device__ void scan_segment(const KArgs &A, const Ctrl &c, Smem &sm, int seg, int &lmin, int &gcnt)
+// Scan entries [lo,hi) of list `src` (nullptr: the identity, ids lo..hi-1)
+// with every warp of this CTA (Alg. 2): eight entries per lane in flight;
+// deg == k -> claim + route (local frontier or global queue); deg > k ->
+// min for the level skip and, when compacting, ballot compaction (Fig. 8(c))
+// into dst[0..) with a shared-memory cursor.  No block sync, no global atomics.
+__device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_t *src, int64_t lo,
+                           int64_t hi, int32_t *dst, int &lmin, int &gcnt)
 {
     const int k = c.k;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const int64_t base = (int64_t)seg * A.seg_R;
-    int64_t len;
-    if (c.src_sel < 0) len = max((int64_t)0, min(A.seg_R, A.n - base));
-    else len = ld_cg_i32(A.seg_len[c.src_sel] + seg);
-    const int32_t *src = c.src_sel < 0 ? nullptr : A.alive[c.src_sel] + base;
-    int32_t *dst = c.compact ? A.alive[c.dst_sel] + base : nullptr;
-    int kcur = 0;
     constexpr int CH = 32 * kScanItems;
-    for (int64_t off = 0; off < len; off += CH) {
+    for (int64_t off = lo + (int64_t)wib * CH; off < hi; off += (int64_t)kWarps * CH) {
         int32_t vv[kScanItems], dd[kScanItems];
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
             const int64_t idx = off + j * 32 + lane;
             vv[j] = -1;
-            if (idx < len) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)(base + idx);
+            if (idx < hi) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)idx;
         }
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_cg_i32(A.deg + vv[j]) : -1;
-        unsigned wm = 0;
+        unsigned wm = 0, km = 0;
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
             if (dd[j] == k) { if (claim(A, vv[j])) wm |= 1u << j; }
-            else if (dd[j] > k) lmin = min(lmin, dd[j]);
+            else if (dd[j] > k) { lmin = min(lmin, dd[j]); km |= 1u << j; }
         }
         if (dst) {
+            int mine = __popc(km), incl = mine;
 #pragma unroll
-            for (int j = 0; j < kScanItems; j++) {
-                const bool keep = dd[j] > k;
-                const unsigned b = __ballot_sync(kFull, keep);
-                if (keep) dst[kcur + __popc(b & lanemask_lt())] = vv[j];
-                kcur += __popc(b);
+            for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += t;
             }
+            const int tot = __shfl_sync(kFull, incl, 31);
+            int pos = 0;
+            if (lane == 31 && tot) pos = atomicAdd(&sm.kcur, tot);
+            pos = __shfl_sync(kFull, pos, 31) + incl - mine;
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++)
+                if ((km >> j) & 1u) dst[pos++] = vv[j];
         }
         if (__any_sync(kFull, wm != 0)) {
             // row bounds of every claimed vertex first (all loads in flight), then route
@@ -630,9 +635,40 @@ __device__ void scan_segment(const KArgs &A, const Ctrl &c, Smem &sm, int seg, i
             }
         }
     }
-    if (lane == 0 && dst) {
-        A.seg_len[c.dst_sel][seg] = kcur;
-        if (kcur) atomicAdd(&A.S->alive_out, (unsigned long long)kcur);
+}
+
+// Source layout: identity (src_sel < 0), one contiguous run (src_single) or
+// per-CTA segments.  Grid mode: CTA b scans its share and compacts into its
+// own segment b.  Solo mode: CTA 0 scans everything and compacts into one
+// contiguous run (segment 0).
+__device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk, int &lmin,
+                           int &gcnt)
+{
+    const bool solo = (nblk == 1);
+    const int32_t *srcb = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
+    int32_t *dstb = c.compact ? A.alive[c.dst_sel] : nullptr;
+    const int dseg = solo ? 0 : bid;
+    if (threadIdx.x == 0) sm.kcur = 0;
+    __syncthreads();
+    int32_t *dst = dstb ? dstb + (int64_t)dseg * A.seg_R : nullptr;
+    if (c.src_sel < 0 || c.src_single) {
+        // contiguous source of c.src_len entries: an even slice per CTA
+        const int64_t L = c.src_len;
+        const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
+        scan_range(A, c, sm, srcb, lo, hi, dst, lmin, gcnt);
+    } else if (!solo) {
+        const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + bid);
+        scan_range(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt);
+    } else {
+        for (int b = 0; b < A.nseg; b++) {
+            const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
+            if (len) scan_range(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, gcnt);
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && dstb) {
+        A.seg_len[c.dst_sel][dseg] = sm.kcur;
+        if (sm.kcur) atomicAdd(&A.S->alive_out, (unsigned long long)sm.kcur);
     }
 }
 
@@ -648,9 +684,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
     }
     __syncthreads();
-    // warp w of CTA b owns segment b*kWarps + w; a solo CTA takes all of them
-    for (int seg = bid * kWarps + wib; seg < A.nseg; seg += nblk * kWarps)
-        scan_segment(A, c, sm, seg, lmin, gcnt);
+    level_scan(A, c, sm, bid, nblk, lmin, gcnt);
     __syncthreads();
     cta_time(A, c, 1);
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
@@ -723,6 +757,7 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
             if (c.compact) {
                 c.alive_sel = c.dst_sel;
                 c.alive_len = (int64_t)sn.alive_out;
+                c.alive_single = c.solo;  // a solo scan compacts into one run
                 c.st_compact++;
             }
         } else {
@@ -754,10 +789,13 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         c.k = next_k;
         c.level++;
         c.src_sel = c.alive_sel;
+        c.src_single = c.alive_single;
         c.src_len = src_len;
         c.compact = compact ? 1 : 0;
         c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
         c.solo = src_len <= (int64_t)p.solo_scan;
+        // a solo scan of a segmented list gathers it into one run for next time
+        if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
         c.ord_lvl0 = removed;
     }
 }

@@ -161,7 +161,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     if (bps > di.occ) bps = di.occ;
     if (bps < 1) return KCORE_EUNSUPPORTED;
     const int grid = di.sms * bps;
-    if (grid * kWarps > kMaxSeg) return KCORE_EUNSUPPORTED;
+    if (grid > kMaxSeg) return KCORE_EUNSUPPORTED;
     int solo = default_solo_arcs(), solo_scan = default_solo_scan();
     if (opt && opt->solo_arcs > 0) solo = opt->solo_arcs;
     if (opt && opt->solo_arcs < 0) solo = 0;
@@ -201,7 +201,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.alive[1] = cv.alive1;
     A.seg_len[0] = cv.seg0;
     A.seg_len[1] = cv.seg1;
-    A.nseg = grid * kWarps;
+    A.nseg = grid;
     A.seg_R = (n + A.nseg - 1) / A.nseg;
     A.pad = 0;
     A.S = cv.S;
