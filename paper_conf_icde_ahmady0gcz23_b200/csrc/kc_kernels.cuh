@@ -529,18 +529,25 @@ __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
     for (int w = threadIdx.x; w < kBloomWords; w += kBlock) sm.bloom[w] = 0u;
     __syncthreads();
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const int nseg = c.src_single ? 1 : A.nseg;
-    for (int b = wib; b < nseg; b += kWarps) {  // one warp per segment
-        const int32_t *src = A.alive[c.src_sel] + (int64_t)b * A.seg_R;
-        const int64_t len = c.src_single ? c.src_len : ld_cg_i32(A.seg_len[c.src_sel] + b);
-        const int64_t step = c.src_single ? (int64_t)kBlock : 32;
-        for (int64_t i = c.src_single ? threadIdx.x : lane; i < len; i += step) {
+    if (c.src_single) {  // one contiguous run: every thread strides it
+        const int32_t *src = A.alive[c.src_sel];
+        for (int64_t i = threadIdx.x; i < c.src_len; i += kBlock) {
             const uint32_t v = (uint32_t)ld_cg_i32(src + i);
             const uint32_t h1 = bloom_h1(v), h2 = bloom_h2(v);
             atomicOr(&sm.bloom[h1 >> 5], 1u << (h1 & 31));
             atomicOr(&sm.bloom[h2 >> 5], 1u << (h2 & 31));
         }
-        if (c.src_single) break;
+    } else {  // per-CTA segments: one warp per segment
+        for (int b = wib; b < A.nseg; b += kWarps) {
+            const int32_t *src = A.alive[c.src_sel] + (int64_t)b * A.seg_R;
+            const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
+            for (int64_t i = lane; i < len; i += 32) {
+                const uint32_t v = (uint32_t)ld_cg_i32(src + i);
+                const uint32_t h1 = bloom_h1(v), h2 = bloom_h2(v);
+                atomicOr(&sm.bloom[h1 >> 5], 1u << (h1 & 31));
+                atomicOr(&sm.bloom[h2 >> 5], 1u << (h2 & 31));
+            }
+        }
     }
     __syncthreads();
     if (threadIdx.x == 0) { sm.bloom_level = c.level; sm.bloom_on = 1; }
