@@ -49,10 +49,12 @@ constexpr int kBlock = 768;
 constexpr int kWarps = kBlock / 32;
 constexpr int kScanItems = 8;        // alive-list entries per lane per warp step
 constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)
-constexpr int kHub = 8192;           // arcs; bigger vertices go to the global queue
+// CTA-local routing budgets (arcs), chosen per level from the size of the
+// previous level: light levels keep their BFS local, heavy ones go grid-wide.
+constexpr int kLightLevelArcs = 4 << 20;
+constexpr int kHubLight = 32768, kSubLight = 32768, kPhaseLight = 262144;
+constexpr int kHubHeavy = 8192, kSubHeavy = 8192, kPhaseHeavy = 16384;
 constexpr int kGStage = 64;          // per-warp global-queue stage (any size; flushed 32 at a time)
-constexpr int kLArcs = 8192;         // arc budget of one CTA-local sub-round
-constexpr int kLPhaseArcs = 16384;   // arc budget of all local sub-rounds of one phase
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -66,7 +68,9 @@ struct Ctrl {
     int32_t phase, solo, k, level_min;
     int32_t compact, src_sel, dst_sel, alive_sel;
     int32_t src_single, alive_single;  // 1: the list is one contiguous run in segment 0
-    int32_t pad0, pad1;
+    int32_t light;                     // budgets of this level (see kLightLevelArcs)
+    int32_t pad1;
+    int64_t arcs_lvl0;                 // arcs walked when the level began
     int64_t src_len, alive_len;
     int64_t s, e, as, ae;          // HUB: global-queue slots [s,e), arcs [as,ae)
     int64_t gq_cnt, gq_arc;        // global queue consumed so far
@@ -79,6 +83,7 @@ struct Ctrl {
 static_assert(sizeof(Ctrl) % 16 == 0, "Ctrl is copied as int4");
 
 struct Snap {
+    unsigned long long arcs;       // arcs walked so far
     unsigned long long gq;         // packed global-queue tail
     unsigned long long ord;        // order tail (= removed vertices)
     unsigned long long alive_out;  // compaction output length
@@ -140,6 +145,7 @@ struct Smem {
     int32_t removed;     // vertices removed by this CTA this phase (order not recorded)
     int32_t fit;         // unused
     int32_t kcur;        // scan: compaction cursor within the current segment
+    int32_t bud_hub, bud_sub, bud_phase, bud_pad;  // routing budgets of this phase
     unsigned long long scan_q2[kWarps];
     unsigned long long tot_q2, base_g, base_w;
     int32_t gv[kWarps][kGStage];
@@ -331,7 +337,7 @@ __device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, boo
             atomicAdd(&sm.removed, __popc(b));
         }
     }
-    const bool cand = won && dv > 0 && dv <= kHub;
+    const bool cand = won && dv > 0 && dv <= sm.bud_hub;
     const unsigned bc = __ballot_sync(kFull, cand);
     bool wantl = false;
     int lbase = 0;
@@ -344,9 +350,9 @@ __device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, boo
         int ok = 0;
         if (lane == lead) {
             oa = atomicAdd(&sm.larc[nx], sumd);
-            if (oa + sumd <= kLArcs) {
+            if (oa + sumd <= sm.bud_sub) {
                 const int op = atomicAdd(&sm.lphase, sumd);
-                if (op + sumd <= kLPhaseArcs) { ok = 1; lbase = atomicAdd(&sm.lcnt[nx], __popc(bc)); }
+                if (op + sumd <= sm.bud_phase) { ok = 1; lbase = atomicAdd(&sm.lcnt[nx], __popc(bc)); }
             }
         }
         ok = __shfl_sync(kFull, ok, lead);
@@ -605,7 +611,8 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
         unsigned wm = 0, km = 0;
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
-            if (dd[j] == k) { if (claim(A, vv[j])) wm |= 1u << j; }
+            // at k = 0 the frontier is the isolated vertices: nothing can race for them
+            if (dd[j] == k) { if (k == 0 || claim(A, vv[j])) wm |= 1u << j; }
             else if (dd[j] > k) { lmin = min(lmin, dd[j]); km |= 1u << j; }
         }
         if (dst) {
@@ -689,6 +696,9 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
+        sm.bud_hub = c.light ? kHubLight : kHubHeavy;
+        sm.bud_sub = c.light ? kSubLight : kSubHeavy;
+        sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
@@ -720,6 +730,9 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
+        sm.bud_hub = c.light ? kHubLight : kHubHeavy;
+        sm.bud_sub = c.light ? kSubLight : kSubHeavy;
+        sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
     }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
@@ -779,6 +792,7 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         }
         // level end
         if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
+        c.light = ((int64_t)sn.arcs - c.arcs_lvl0) < kLightLevelArcs;
         if (removed >= p.n) {
             c.phase = PH_DONE;
             c.solo = 0;
@@ -804,6 +818,7 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         // a solo scan of a segmented list gathers it into one run for next time
         if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
         c.ord_lvl0 = removed;
+        c.arcs_lvl0 = (int64_t)sn.arcs;
     }
 }
 
@@ -811,6 +826,7 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
 __device__ __forceinline__ Snap take_snapshot(State *S)
 {
     Snap sn;
+    sn.arcs = ld_relaxed_u64(&S->arcs_walked);
     sn.gq = ld_relaxed_u64(&S->gq_tail);
     sn.ord = ld_relaxed_u64(&S->ord_tail);
     sn.alive_out = ld_relaxed_u64(&S->alive_out);
@@ -857,6 +873,7 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
             while (ld_acquire_u32(&S->bar_gen) == gen) {
             }
             const Snap *ps = &S->snap[(gen + 1u) & 1u];
+            sn.arcs = ld_relaxed_u64(&ps->arcs);
             sn.gq = ld_relaxed_u64(&ps->gq);
             sn.ord = ld_relaxed_u64(&ps->ord);
             sn.alive_out = ld_relaxed_u64(&ps->alive_out);
@@ -903,6 +920,7 @@ __device__ __forceinline__ void init_ctrl(Ctrl &z)
     z.level_min = INT_MAX;
     z.alive_sel = -1;
     z.src_sel = -1;
+    z.light = 1;
 }
 
 __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
