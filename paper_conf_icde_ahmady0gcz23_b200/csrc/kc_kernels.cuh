@@ -71,6 +71,7 @@ struct Ctrl {
     int32_t light;                     // budgets of this level (see kLightLevelArcs)
     int32_t pad1;
     int64_t arcs_lvl0;                 // arcs walked when the level began
+    int64_t pad2;
     int64_t src_len, alive_len;
     int64_t s, e, as, ae;          // HUB: global-queue slots [s,e), arcs [as,ae)
     int64_t gq_cnt, gq_arc;        // global queue consumed so far
