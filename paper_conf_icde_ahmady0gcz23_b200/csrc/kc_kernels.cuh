@@ -793,7 +793,8 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         }
         // level end
         if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
-        c.light = ((int64_t)sn.arcs - c.arcs_lvl0) < kLightLevelArcs;
+        c.light = 0;  // adaptive budgets disabled: misjudge level jumps
+        (void)kLightLevelArcs;
         if (removed >= p.n) {
             c.phase = PH_DONE;
             c.solo = 0;
@@ -921,7 +922,7 @@ __device__ __forceinline__ void init_ctrl(Ctrl &z)
     z.level_min = INT_MAX;
     z.alive_sel = -1;
     z.src_sel = -1;
-    z.light = 1;
+    z.light = 0;
 }
 
 __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
