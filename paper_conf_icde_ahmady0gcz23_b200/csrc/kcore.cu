@@ -192,7 +192,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.rowptr = rowptr;
     A.colidx = colidx;
     A.deg = core_out;
-    A.order = cv.order;
+    A.order = (opt && opt->order_out) ? cv.order : nullptr;  // record the peel order only on request
     A.claimed = cv.claimed;
     A.gq_v = cv.gq_v;
     A.gq_beg = cv.gq_beg;
