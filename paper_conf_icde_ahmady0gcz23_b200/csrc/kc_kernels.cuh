@@ -52,7 +52,9 @@ constexpr int kLCap = kBlock;        // local frontier capacity (one entry per t
 constexpr int kChunk = 4096;         // max arcs of one pool entry (hubs are split)
 constexpr int kSub = 8192;           // arc budget of one CTA-local sub-round
 constexpr int kPStage = 64;          // per-warp pool stage (vertices)
-constexpr int kClaim = 16;           // pool entries claimed at a time
+constexpr int kClaimMin = 8;         // pool entries claimed at a time: backlog / (2 grid),
+constexpr int kClaimMax = kLCap;     //   clamped to [kClaimMin, kClaimMax]
+constexpr int kMaxLocalRounds = 4;   // then the local frontier goes back to the pool
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -520,10 +522,32 @@ __device__ int64_t local_drain(const KArgs &A, const Ctrl &c, Smem &sm, int cur,
 {
     const int wib = threadIdx.x >> 5;
     int64_t walked = 0;
-    while (true) {
+    for (int round = 0;; round++) {
         __syncthreads();
         const int L = min(sm.lcnt[cur], kLCap);
         if (L == 0) break;
+        if (round == kMaxLocalRounds && c.solo == 0) {
+            // a long local chain: hand the frontier back to the pool so idle
+            // CTAs share it (each warp pushes a slice through its stage)
+            for (int x0 = wib * 32; x0 < L; x0 += kWarps * 32) {
+                const int x = x0 + (threadIdx.x & 31);
+                const bool has = x < L;
+                const unsigned bg = __ballot_sync(kFull, has);
+                if (pcnt + __popc(bg) > kPStage) pool_flush(A, sm, wib, pcnt);
+                if (has) {
+                    const int pos = pcnt + __popc(bg & lanemask_lt());
+                    sm.pv[wib][pos] = sm.lv[cur][x];
+                    sm.pd[wib][pos] = sm.ld[cur][x];
+                    sm.pb[wib][pos] = sm.lb[cur][x];
+                }
+                pcnt += __popc(bg);
+                __syncwarp();
+            }
+            __syncthreads();
+            if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
+            __syncthreads();
+            break;
+        }
         const int64_t dv = threadIdx.x < L ? (int64_t)sm.ld[cur][threadIdx.x] : 0;
         const unsigned long long ex = block_excl_scan(sm, (unsigned long long)dv);
         if (threadIdx.x < L) sm.lpre[threadIdx.x] = (int64_t)ex;
@@ -692,7 +716,10 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
             unsigned long long cl = ld_acquire_u64(&S->pool_claim);
             const unsigned long long tl = ld_acquire_u64(&S->pool_tail);
             while (cl < tl) {
-                const unsigned long long want = min(cl + (unsigned long long)kClaim, tl);
+                unsigned long long J = (tl - cl) / (2ULL * (unsigned long long)nblk);
+                J = J < (unsigned long long)kClaimMin ? (unsigned long long)kClaimMin
+                                                      : (J > (unsigned long long)kClaimMax ? (unsigned long long)kClaimMax : J);
+                const unsigned long long want = min(cl + J, tl);
                 const unsigned long long got = atomicCAS(&S->pool_claim, cl, want);
                 if (got == cl) { c0 = (int64_t)cl; c1 = (int64_t)want; break; }
                 cl = got;

@@ -42,9 +42,9 @@ def test_strerror_and_version():
 
 
 def test_workspace_size_scales_linearly():
-    a = kc.kcore_workspace_size(1 << 20)
-    b = kc.kcore_workspace_size(1 << 21)
-    assert 30 * (1 << 20) <= a <= 36 * (1 << 20) + 8192
+    a = kc.kcore_workspace_size(1 << 20, 1 << 24)
+    b = kc.kcore_workspace_size(1 << 21, 1 << 24)
+    assert 26 * (1 << 20) <= a <= 40 * (1 << 20) + 65536
     assert b > a
 
 

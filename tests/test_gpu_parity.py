@@ -254,7 +254,7 @@ def test_caller_workspace_and_stream():
     rp, ci = kcgen.generate_host(kcgen.rmat(12, 16, seed=4))
     ref = oracle.bz_core(rp, ci)
     r, c = _to_dev(rp, ci)
-    ws = torch.empty(kc.kcore_workspace_size(rp.size - 1), dtype=torch.uint8, device=DEV)
+    ws = torch.empty(kc.kcore_workspace_size(rp.size - 1, ci.size), dtype=torch.uint8, device=DEV)
     s = torch.cuda.Stream()
     with torch.cuda.stream(s):
         out = kc.kcore_decompose(r, c, workspace=ws)

@@ -12,7 +12,7 @@ for a in sys.argv[2:]:
     k, v = a.split('=')
     kw[k] = int(v)
 r, c = kcgen.generate_device(kcgen.CONFIGS[name])
-ws = torch.empty(kc.kcore_workspace_size(r.numel() - 1), dtype=torch.uint8, device='cuda')
+ws = torch.empty(kc.kcore_workspace_size(r.numel() - 1, c.numel()), dtype=torch.uint8, device='cuda')
 for _ in range(2):
     core, st = kc.kcore_decompose(r, c, workspace=ws, stats=True, **kw)
 print(name, kw, st)
