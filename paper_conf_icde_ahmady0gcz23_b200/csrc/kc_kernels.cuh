@@ -55,6 +55,7 @@ constexpr int kPStage = 64;          // per-warp pool stage (vertices)
 constexpr int kClaimMin = 8;         // pool entries claimed at a time: backlog / (2 grid),
 constexpr int kClaimMax = kLCap;     //   clamped to [kClaimMin, kClaimMax]
 constexpr int kMaxLocalRounds = 4;   // then the local frontier goes back to the pool
+constexpr int kSoloBail = 32;        // a solo level with more pending pool entries goes grid-wide
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -68,14 +69,15 @@ struct Ctrl {
     int32_t phase, solo, k, level_min;
     int32_t compact, src_sel, dst_sel, alive_sel;
     int32_t src_single, alive_single;  // 1: the list is one contiguous run in segment 0
-    int32_t pad0, pad1;
+    int32_t cont;                      // 1: the level's scan is done, only the pool is left
+    int32_t pad1;
     int64_t src_len, alive_len;
     int64_t scan_target;               // scans_done value that ends the current level
     int64_t ord_lvl0;                  // removed count when the level began
     int64_t level;                     // level index (for the Bloom cache)
     int64_t st_levels, st_phases, st_solo, st_bar, st_scanned, st_compact, st_pool;
     int32_t st_kmax, st_pad;
-    int64_t pad2;
+    int64_t alive_carry;               // compaction output already counted (solo bail-out)
 };
 
 static_assert(sizeof(Ctrl) % 16 == 0, "Ctrl is copied as int4");
@@ -526,7 +528,7 @@ __device__ int64_t local_drain(const KArgs &A, const Ctrl &c, Smem &sm, int cur,
         __syncthreads();
         const int L = min(sm.lcnt[cur], kLCap);
         if (L == 0) break;
-        if (round == kMaxLocalRounds && c.solo == 0) {
+        if (round == kMaxLocalRounds) {
             // a long local chain: hand the frontier back to the pool so idle
             // CTAs share it (each warp pushes a slice through its stage)
             for (int x0 = wib * 32; x0 < L; x0 += kWarps * 32) {
@@ -687,29 +689,42 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
 
 // One level (Alg. 1 round k): scan, drain the local frontier, then share the
 // pool until every CTA has scanned and every pool entry is processed.
-__device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+// c.cont: the scan was done by a solo CTA that bailed out; only the pool is
+// left.  A solo CTA (nblk == 1) bails out when its pool backlog is large and
+// returns true (the grid then finishes the level).
+__device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
 {
     const int wib = threadIdx.x >> 5;
     State *S = A.S;
     int lmin = INT_MAX, pcnt = 0;
+    int64_t walked = 0;
     cta_time(A, c, 0);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.removed = 0; sm.lvl_arcs = 0;
     }
     __syncthreads();
-    level_scan(A, c, sm, bid, nblk, lmin, pcnt);
-    cta_time(A, c, 1);
-    int64_t walked = local_drain(A, c, sm, 0, lmin, pcnt);
-    pool_flush(A, sm, wib, pcnt);
-    __syncthreads();
+    if (!c.cont) {
+        level_scan(A, c, sm, bid, nblk, lmin, pcnt);
+        cta_time(A, c, 1);
+        walked = local_drain(A, c, sm, 0, lmin, pcnt);
+        pool_flush(A, sm, wib, pcnt);
+        __syncthreads();
+    }
     cta_time(A, c, 2);
     if (threadIdx.x == 0) {
         __threadfence();
         atomicAdd(&S->scans_done, 1ULL);
+        sm.done = 0;
+        if (nblk == 1) {
+            const unsigned long long pend = ld_acquire_u64(&S->pool_tail) - ld_acquire_u64(&S->pool_done);
+            if (pend > (unsigned long long)kSoloBail) sm.done = 2;
+        }
     }
+    __syncthreads();
+    const bool bail = sm.done == 2;
     // pool loop: claim, copy into the local frontier, drain, report
-    while (true) {
+    while (!bail) {
         if (threadIdx.x == 0) {
             int64_t c0 = -1, c1 = -1;
             int done = 0;
@@ -762,6 +777,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         if (sm.removed) atomicAdd(&S->ord_tail, (unsigned long long)sm.removed);
     }
     block_min_atomic(sm, lmin, &S->min_next);
+    return bail;
 }
 
 // ---------------------------------------------------------------- control
@@ -783,8 +799,8 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p, i
         c.st_pool = (int64_t)sn.pool;
         if (c.compact) {
             c.alive_sel = c.dst_sel;
-            c.alive_len = (int64_t)sn.alive_out;
-            c.alive_single = c.solo;  // a solo scan compacts into one run
+            c.alive_len = (int64_t)sn.alive_out + c.alive_carry;
+            c.alive_single = c.solo || c.cont;  // a solo scan compacts into one run
             c.st_compact++;
         }
         if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
@@ -799,6 +815,8 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p, i
     const int64_t live = p.n - removed;
     const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
     c.phase = PH_LEVEL;
+    c.cont = 0;
+    c.alive_carry = 0;
     c.k = next_k;
     c.level++;
     c.src_sel = c.alive_sel;
@@ -880,7 +898,22 @@ __device__ void solo_run(const KArgs &A, Smem &sm, const Params &p)
     State *S = A.S;
     while (true) {
         const Ctrl c = sm.ctrl;
-        phase_level(A, c, sm, 0, 1);  // ends with __syncthreads (block_min_atomic)
+        const bool bail = phase_level(A, c, sm, 0, 1);  // ends with __syncthreads
+        if (bail) {  // the level's pool is too big for one CTA: the grid finishes it
+            if (threadIdx.x == 0) {
+                // fold this partial level's counters into the control state: the
+                // barrier that follows resets them before the grid continues
+                __threadfence();
+                const Snap sn = take_snapshot(S);
+                sm.ctrl.level_min = min(sm.ctrl.level_min, sn.min);
+                sm.ctrl.alive_carry = (int64_t)sn.alive_out;
+                sm.ctrl.cont = 1;
+                sm.ctrl.solo = 0;
+                sm.ctrl.scan_target += gridDim.x;
+            }
+            __syncthreads();
+            break;
+        }
         if (threadIdx.x == 0) {
             __threadfence();
             const Snap sn = take_snapshot(S);
