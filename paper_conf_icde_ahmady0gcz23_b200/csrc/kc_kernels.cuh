@@ -724,12 +724,14 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     __syncthreads();
     const bool bail = sm.done == 2;
     // pool loop: claim, copy into the local frontier, drain, report
-    while (!bail) {
+    bool bailed = bail;
+    while (!bailed) {
         if (threadIdx.x == 0) {
             int64_t c0 = -1, c1 = -1;
             int done = 0;
             unsigned long long cl = ld_acquire_u64(&S->pool_claim);
             const unsigned long long tl = ld_acquire_u64(&S->pool_tail);
+            if (nblk == 1 && tl - cl > (unsigned long long)kSoloBail) { cl = tl; done = 2; }
             while (cl < tl) {
                 unsigned long long J = (tl - cl) / (2ULL * (unsigned long long)nblk);
                 J = J < (unsigned long long)kClaimMin ? (unsigned long long)kClaimMin
@@ -739,7 +741,7 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
                 if (got == cl) { c0 = (int64_t)cl; c1 = (int64_t)want; break; }
                 cl = got;
             }
-            if (c0 < 0) {
+            if (c0 < 0 && done == 0) {
                 const unsigned long long dn = ld_acquire_u64(&S->pool_done);
                 const unsigned long long sd = ld_acquire_u64(&S->scans_done);
                 const unsigned long long t2 = ld_acquire_u64(&S->pool_tail);
@@ -751,6 +753,7 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
             sm.done = done;
         }
         __syncthreads();
+        if (sm.done == 2) { bailed = true; break; }
         if (sm.done) break;
         const int64_t c0 = sm.c0, c1 = sm.c1;
         if (c0 < 0) continue;
@@ -777,7 +780,7 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         if (sm.removed) atomicAdd(&S->ord_tail, (unsigned long long)sm.removed);
     }
     block_min_atomic(sm, lmin, &S->min_next);
-    return bail;
+    return bailed;
 }
 
 // ---------------------------------------------------------------- control
