@@ -1,4 +1,4 @@
-// kc_kernels.cuh -- sm_100a kernels of the k-core hot path (v4).
+// kc_kernels.cuh -- sm_100a kernels of the k-core hot path (v5).
 //
 // One call = one persistent cooperative kernel (k_persistent), one CTA per SM,
 // running the whole decomposition as a device-resident state machine.  Per
@@ -18,11 +18,14 @@
 //                             frontier (or the pool)
 //               old <= k   -> atomicAdd(&deg[u],1)  (restore, Fig. 6)
 //               else       -> min_next = min(min_next, old-1)          (level skip)
-//   pool   a CTA with no local work claims pool entries (each <= kChunk arcs,
-//          hubs are pre-split), copies them into its local frontier and drains
-//          them the same way -- asynchronous work sharing, no sub-round
-//          barrier.  The level ends when every CTA has finished its scan and
-//          the pool's done count equals its tail.
+//   pool   vertices too big for a CTA-local sub-round, or overflowing it, go
+//          to a global pool (one packed atomic reserves entries and their
+//          range in the pool's ARC space).  A CTA with no local work claims a
+//          range of pool arcs (CAS, never past the reserved arcs) and walks it
+//          with all its warps, arc-balanced (hubs are shared by many CTAs),
+//          then drains the local frontier that produced -- asynchronous work
+//          sharing, no sub-round barrier.  The level ends when every CTA has
+//          finished its scan and the pool's done arcs equal its reserved arcs.
 //   level end: k <- max(k+1, min_next)  (Alg. 1 l.9 does k+1; reading R5)
 //
 // Scans and drains of one level run concurrently in different CTAs, so a
@@ -49,13 +52,12 @@ constexpr int kBlock = 768;
 constexpr int kWarps = kBlock / 32;
 constexpr int kScanItems = 8;        // alive-list entries per lane per warp step
 constexpr int kLCap = kBlock;        // local frontier capacity (one entry per thread in the prefix)
-constexpr int kChunk = 4096;         // max arcs of one pool entry (hubs are split)
 constexpr int kSub = 8192;           // arc budget of one CTA-local sub-round
 constexpr int kPStage = 64;          // per-warp pool stage (vertices)
-constexpr int kClaimMin = 8;         // pool entries claimed at a time: backlog / (2 grid),
-constexpr int kClaimMax = kLCap;     //   clamped to [kClaimMin, kClaimMax]
+constexpr int kClaimMin = 4096;      // pool ARCS claimed at a time: backlog / (2 grid),
+constexpr int kClaimMax = 1 << 17;   //   clamped to [kClaimMin, kClaimMax]
 constexpr int kMaxLocalRounds = 4;   // then the local frontier goes back to the pool
-constexpr int kSoloBail = 32;        // a solo level with more pending pool entries goes grid-wide
+constexpr int kSoloBail = 65536;     // a solo level with more pending pool arcs goes grid-wide
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -102,9 +104,9 @@ struct State {
     alignas(128) unsigned long long ord_tail;   // removed vertices (order slots if recorded)
     alignas(128) unsigned long long alive_out;  // compaction output length
     alignas(128) int32_t min_next;              // atomicMin target
-    alignas(128) unsigned long long pool_tail;  // pool entries reserved
-    alignas(128) unsigned long long pool_claim; // pool entries claimed
-    alignas(128) unsigned long long pool_done;  // pool entries fully processed
+    alignas(128) unsigned long long pool_tail;  // packed (entries << 33) | arcs reserved
+    alignas(128) unsigned long long pool_claim; // pool arcs claimed
+    alignas(128) unsigned long long pool_done;  // pool arcs fully processed
     alignas(128) unsigned long long scans_done; // CTA scans finished (monotone)
     alignas(128) uint32_t bar_count;            // grid barrier arrivals (monotone)
     alignas(128) uint32_t bar_gen;              // grid barrier generation
@@ -124,9 +126,10 @@ struct KArgs {
     int32_t *deg;         // == core_out
     int32_t *order;       // removal order, or nullptr when not requested
     uint32_t *claimed;    // claim bit per vertex
-    int32_t *pool_v;      // pool entry: vertex,
-    int64_t *pool_beg;    //   first arc of the chunk,
-    int32_t *pool_len;    //   arcs in the chunk (0 = not yet published; zeroed at init)
+    int32_t *pool_v;      // pool entry j: vertex,
+    int64_t *pool_beg;    //   its first arc in colidx,
+    int64_t *pool_P;      //   its first arc in the pool's arc space (prefix),
+    int32_t *pool_len;    //   its arcs (0 = not yet published; zeroed at init)
     int64_t pool_cap;
     int32_t *alive[2];    // alive lists, one segment per CTA
     int32_t *seg_len[2];  // entries of segment b in alive[x]: seg_len[x][b]
@@ -152,7 +155,8 @@ struct Smem {
     unsigned long long scan_q[kWarps];
     unsigned long long tot_q;
     int32_t red_min[kWarps];
-    int64_t c0, c1;      // claimed pool entries
+    int64_t c0, c1;      // claimed pool arcs
+    int64_t cnt;         // pool entries reserved when they were claimed
     int32_t done, pad3;
     int64_t lvl_arcs;    // arcs this CTA walked in the current level
     int64_t bloom_level;
@@ -261,50 +265,48 @@ __device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
 }
 
 // ------------------------------------------------------------- the pool
-// Flush this warp's pool stage: every vertex becomes ceil(d/kChunk) entries;
-// one atomic reserves them all.  Entries are published by writing their
+// Flush this warp's pool stage: one packed atomic reserves the entries and
+// their range in the pool's arc space; entries are published by writing their
 // length last, after a fence (consumers spin until it is non-zero).
 __device__ __noinline__ void pool_flush(const KArgs &A, Smem &sm, int wib, int &pcnt)
 {
     const int lane = threadIdx.x & 31;
     if (pcnt == 0) return;
     __syncwarp();
-    int ch[2], pre[2];
-    int carry = 0;
+    int64_t dd[2], pre[2];
+    int64_t carry = 0;
 #pragma unroll
     for (int h = 0; h < 2; h++) {
         const int x = h * 32 + lane;
-        ch[h] = x < pcnt ? (sm.pd[wib][x] + kChunk - 1) / kChunk : 0;
-        int incl = ch[h];
+        dd[h] = x < pcnt ? (int64_t)sm.pd[wib][x] : 0;
+        int64_t incl = dd[h];
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
-            const int t = __shfl_up_sync(kFull, incl, o);
+            const int64_t t = __shfl_up_sync(kFull, incl, o);
             if (lane >= o) incl += t;
         }
-        pre[h] = carry + incl - ch[h];
+        pre[h] = carry + incl - dd[h];
         carry += __shfl_sync(kFull, incl, 31);
     }
     unsigned long long base = 0;
-    if (lane == 0) base = atomicAdd(&A.S->pool_tail, (unsigned long long)carry);
+    if (lane == 0)
+        base = atomicAdd(&A.S->pool_tail, ((unsigned long long)pcnt << kArcBits) | (unsigned long long)carry);
     base = __shfl_sync(kFull, base, 0);
+    const int64_t bc = (int64_t)(base >> kArcBits), ba = (int64_t)(base & kArcMask);
 #pragma unroll
     for (int h = 0; h < 2; h++) {
         const int x = h * 32 + lane;
-        if (x >= pcnt) continue;
-        for (int c = 0; c < ch[h]; c++) {
-            const int64_t slot = (int64_t)base + pre[h] + c;
-            A.pool_v[slot] = sm.pv[wib][x];
-            A.pool_beg[slot] = sm.pb[wib][x] + (int64_t)c * kChunk;
+        if (x < pcnt) {
+            A.pool_v[bc + x] = sm.pv[wib][x];
+            A.pool_beg[bc + x] = sm.pb[wib][x];
+            A.pool_P[bc + x] = ba + pre[h];
         }
     }
     __threadfence();
 #pragma unroll
     for (int h = 0; h < 2; h++) {
         const int x = h * 32 + lane;
-        if (x >= pcnt) continue;
-        const int d = sm.pd[wib][x];
-        for (int c = 0; c < ch[h]; c++)
-            A.pool_len[(int64_t)base + pre[h] + c] = min(kChunk, d - c * kChunk);
+        if (x < pcnt) A.pool_len[bc + x] = (int32_t)dd[h];
     }
     __syncwarp();
     pcnt = 0;
@@ -434,6 +436,93 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
         else if (lane == 31) nxt = sm.lpre[j + 1];
         const int64_t limit = min(a1, __shfl_sync(kFull, nxt, 31));
         const int64_t bmq = wbeg - wq;  // colidx index of arc x in this entry = bmq + x
+        while (a < limit) {
+            const int64_t rq = wq - a;
+            const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
+            const int32_t lim = (int32_t)min((int64_t)kBatch, limit - a);
+            int32_t u[kUnroll];
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) {
+                const int32_t my = r * 32 + lane;
+                int pos = 0;
+#pragma unroll
+                for (int bs = 16; bs >= 1; bs >>= 1) {
+                    const int32_t q = __shfl_sync(kFull, q32, pos + bs);
+                    if (q <= my) pos += bs;
+                }
+                const int64_t off = __shfl_sync(kFull, bmq, pos);
+                u[r] = (my < lim) ? ld_stream_i32(A.colidx + off + a + my) : -1;
+            }
+            if (use_bloom) {
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++)
+                    if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
+            }
+            int32_t d[kUnroll];
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) d[r] = u[r] >= 0 ? ld_cg_i32(A.deg + u[r]) : -1;
+            int old[kUnroll];
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
+            unsigned hm = 0;
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) {
+                if (old[r] == k + 1) hm |= 1u << r;
+                else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
+                else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
+            }
+            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, pcnt);
+            a += kBatch;
+        }
+        a = limit;
+        i += 32;
+    }
+}
+
+// Pool entry j (spinning until it is published): arc-space start, length, row begin.
+__device__ __forceinline__ int32_t pool_entry(const KArgs &A, int64_t j, int64_t &P, int64_t &beg)
+{
+    int32_t len;
+    while ((len = ld_acquire_i32(A.pool_len + j)) == 0) {
+    }
+    P = ld_cg_i64(A.pool_P + j);
+    beg = ld_cg_i64(A.pool_beg + j);
+    return len;
+}
+
+// Walk pool arcs [a0,a1) with one warp (entries [0,cnt) are reserved; every
+// arc below a1 belongs to one of them).  Same window scheme as walk().
+__device__ __forceinline__ void walk_pool(const KArgs &A, Smem &sm, const int k, const int nx, int64_t cnt,
+                                          int64_t a0, int64_t a1, bool use_bloom, int &lmin, int &pcnt)
+{
+    const int lane = threadIdx.x & 31;
+    int64_t lo = 0, hi = cnt;  // first entry: largest j with P(j) <= a0
+    while (true) {
+        const int64_t step = hi - lo > 32 ? (hi - lo + 31) / 32 : 1;
+        const int64_t p = lo + lane * step;
+        bool ok = false;
+        if (p < hi) {
+            int64_t P, beg;
+            pool_entry(A, p, P, beg);
+            ok = P <= a0;
+        }
+        const unsigned b = __ballot_sync(kFull, ok);
+        lo = lo + (31 - __clz(b)) * step;
+        if (step == 1) break;
+        hi = min(hi, lo + step);
+    }
+    int64_t i = lo;
+    int64_t a = a0;
+    while (a < a1) {
+        const int64_t j = i + lane;
+        int64_t wq = LLONG_MAX, wbeg = 0, wend = LLONG_MAX;
+        if (j < cnt) {
+            const int32_t len = pool_entry(A, j, wq, wbeg);
+            wend = wq + len;
+        }
+        const int last = (int)min((int64_t)31, cnt - 1 - i);
+        const int64_t limit = min(a1, __shfl_sync(kFull, wend, last));
+        const int64_t bmq = wbeg - wq;
         while (a < limit) {
             const int64_t rq = wq - a;
             const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
@@ -717,7 +806,7 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         atomicAdd(&S->scans_done, 1ULL);
         sm.done = 0;
         if (nblk == 1) {
-            const unsigned long long pend = ld_acquire_u64(&S->pool_tail) - ld_acquire_u64(&S->pool_done);
+            const unsigned long long pend = (ld_acquire_u64(&S->pool_tail) & kArcMask) - ld_acquire_u64(&S->pool_done);
             if (pend > (unsigned long long)kSoloBail) sm.done = 2;
         }
     }
@@ -729,14 +818,15 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         if (threadIdx.x == 0) {
             int64_t c0 = -1, c1 = -1;
             int done = 0;
+            const unsigned long long tp = ld_acquire_u64(&S->pool_tail);
+            const unsigned long long tcnt = tp >> kArcBits, tarc = tp & kArcMask;
             unsigned long long cl = ld_acquire_u64(&S->pool_claim);
-            const unsigned long long tl = ld_acquire_u64(&S->pool_tail);
-            if (nblk == 1 && tl - cl > (unsigned long long)kSoloBail) { cl = tl; done = 2; }
-            while (cl < tl) {
-                unsigned long long J = (tl - cl) / (2ULL * (unsigned long long)nblk);
+            if (nblk == 1 && tarc - cl > (unsigned long long)kSoloBail) { cl = tarc; done = 2; }
+            while (cl < tarc) {
+                unsigned long long J = (tarc - cl) / (2ULL * (unsigned long long)nblk);
                 J = J < (unsigned long long)kClaimMin ? (unsigned long long)kClaimMin
                                                       : (J > (unsigned long long)kClaimMax ? (unsigned long long)kClaimMax : J);
-                const unsigned long long want = min(cl + J, tl);
+                const unsigned long long want = min(cl + J, tarc);
                 const unsigned long long got = atomicCAS(&S->pool_claim, cl, want);
                 if (got == cl) { c0 = (int64_t)cl; c1 = (int64_t)want; break; }
                 cl = got;
@@ -744,12 +834,13 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
             if (c0 < 0 && done == 0) {
                 const unsigned long long dn = ld_acquire_u64(&S->pool_done);
                 const unsigned long long sd = ld_acquire_u64(&S->scans_done);
-                const unsigned long long t2 = ld_acquire_u64(&S->pool_tail);
+                const unsigned long long t2 = ld_acquire_u64(&S->pool_tail) & kArcMask;
                 if (sd >= (unsigned long long)c.scan_target && dn == t2) done = 1;
                 else __nanosleep(64);
             }
             sm.c0 = c0;
             sm.c1 = c1;
+            sm.cnt = (int64_t)tcnt;
             sm.done = done;
         }
         __syncthreads();
@@ -757,16 +848,18 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         if (sm.done) break;
         const int64_t c0 = sm.c0, c1 = sm.c1;
         if (c0 < 0) continue;
-        const int64_t j = c0 + threadIdx.x;
-        if (j < c1) {
-            int32_t len;
-            while ((len = ld_acquire_i32(A.pool_len + j)) == 0) {
-            }
-            sm.lv[0][threadIdx.x] = A.pool_v[j];
-            sm.ld[0][threadIdx.x] = len;
-            sm.lb[0][threadIdx.x] = A.pool_beg[j];
+        // arc-balanced walk of the claimed pool arcs; hits go to local list 0
+        {
+            const int64_t T = c1 - c0;
+            const bool bl = want_bloom(A, c, sm, T);
+            int64_t C = (T + kWarps - 1) / kWarps;
+            C = ((C + kBatch - 1) / kBatch) * kBatch;
+            const int64_t w0 = c0 + (int64_t)wib * C;
+            if (w0 < c1) walk_pool(A, sm, c.k, 0, sm.cnt, w0, min(w0 + C, c1), bl, lmin, pcnt);
+            walked += T;
+            __syncthreads();
+            if (threadIdx.x == 0) sm.lvl_arcs += T;
         }
-        if (threadIdx.x == 0) { sm.lcnt[0] = (int)(c1 - c0); sm.larc[0] = 0; }
         walked += local_drain(A, c, sm, 0, lmin, pcnt);  // starts with __syncthreads
         pool_flush(A, sm, wib, pcnt);
         __syncthreads();
@@ -840,7 +933,7 @@ __device__ __forceinline__ Snap take_snapshot(State *S)
     Snap sn;
     sn.ord = ld_relaxed_u64(&S->ord_tail);
     sn.alive_out = ld_relaxed_u64(&S->alive_out);
-    sn.pool = ld_relaxed_u64(&S->pool_tail);
+    sn.pool = ld_relaxed_u64(&S->pool_tail) & kArcMask;
     sn.min = ld_relaxed_i32(&S->min_next);
     sn.pad = 0;
     S->alive_out = 0ULL;

@@ -63,7 +63,7 @@ struct Carve {
     int32_t *order;
     uint32_t *claimed;
     int32_t *pool_v, *pool_len;
-    int64_t *pool_beg;
+    int64_t *pool_beg, *pool_P;
     int64_t pool_cap;
     int32_t *alive0, *alive1;
     int32_t *seg0, *seg1;
@@ -84,11 +84,14 @@ size_t carve(void *base, int64_t n, int64_t m, Carve *c)
     t.S = (State *)take(sizeof(State));
     t.order = (int32_t *)take(sizeof(int32_t) * nn);
     t.claimed = (uint32_t *)take(sizeof(uint32_t) * ((nn + 31) / 32));
-    // every vertex enters the pool at most once, as ceil(deg / kChunk) entries
-    t.pool_cap = (int64_t)nn + (m > 0 ? m : 0) / kChunk + 1;
+    // a vertex enters the pool at most once per level phase it is processed in;
+    // with the local-round cap a frontier may be pushed back once: 2n bounds it
+    (void)m;
+    t.pool_cap = 2 * (int64_t)nn + 1024;
     t.pool_v = (int32_t *)take(sizeof(int32_t) * (size_t)t.pool_cap);
     t.pool_len = (int32_t *)take(sizeof(int32_t) * (size_t)t.pool_cap);
     t.pool_beg = (int64_t *)take(sizeof(int64_t) * (size_t)t.pool_cap);
+    t.pool_P = (int64_t *)take(sizeof(int64_t) * (size_t)t.pool_cap);
     t.alive0 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
@@ -200,6 +203,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.pool_v = cv.pool_v;
     A.pool_beg = cv.pool_beg;
     A.pool_len = cv.pool_len;
+    A.pool_P = cv.pool_P;
     A.pool_cap = cv.pool_cap;
     A.alive[0] = cv.alive0;
     A.alive[1] = cv.alive1;
