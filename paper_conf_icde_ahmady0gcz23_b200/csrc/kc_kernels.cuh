@@ -55,9 +55,9 @@ constexpr int kLCap = kBlock;        // local frontier capacity (one entry per t
 constexpr int kSub = 8192;           // arc budget of one CTA-local sub-round
 constexpr int kPStage = 64;          // per-warp pool stage (vertices)
 constexpr int kClaimMin = 4096;      // pool ARCS claimed at a time: backlog / (2 grid),
-constexpr int kClaimMax = 1 << 17;   //   clamped to [kClaimMin, kClaimMax]
+constexpr int kClaimMax = 1 << 19;   //   clamped to [kClaimMin, kClaimMax]
 constexpr int kMaxLocalRounds = 4;   // then the local frontier goes back to the pool
-constexpr int kSoloBail = 65536;     // a solo level with more pending pool arcs goes grid-wide
+constexpr int kSoloBail = 16384;     // a solo level with more pending pool arcs goes grid-wide
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
@@ -157,6 +157,7 @@ struct Smem {
     int32_t red_min[kWarps];
     int64_t c0, c1;      // claimed pool arcs
     int64_t cnt;         // pool entries reserved when they were claimed
+    int64_t backlog;     // unclaimed pool arcs per CTA when they were claimed
     int32_t done, pad3;
     int64_t lvl_arcs;    // arcs this CTA walked in the current level
     int64_t bloom_level;
@@ -841,6 +842,7 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
             sm.c0 = c0;
             sm.c1 = c1;
             sm.cnt = (int64_t)tcnt;
+            sm.backlog = (int64_t)(tarc - (c0 < 0 ? tarc : (unsigned long long)c0)) / nblk;
             sm.done = done;
         }
         __syncthreads();
@@ -851,7 +853,7 @@ __device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         // arc-balanced walk of the claimed pool arcs; hits go to local list 0
         {
             const int64_t T = c1 - c0;
-            const bool bl = want_bloom(A, c, sm, T);
+            const bool bl = want_bloom(A, c, sm, max(T, sm.backlog));
             int64_t C = (T + kWarps - 1) / kWarps;
             C = ((C + kBatch - 1) / kBatch) * kBatch;
             const int64_t w0 = c0 + (int64_t)wib * C;
