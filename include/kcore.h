@@ -98,13 +98,13 @@ typedef struct {
  * call synchronise `stream`). */
 typedef struct {
     int64_t levels;        /* distinct core values peeled (non-empty levels)          */
-    int64_t phases;        /* level phases executed (grid-wide or single-CTA)         */
+    int64_t phases;        /* LEVEL + HUB phases executed (grid-wide or single-CTA)   */
     int64_t solo_phases;   /* of which ran on a single CTA                             */
     int64_t barriers;      /* grid barriers executed                                   */
     int64_t scanned;       /* sum over levels of scanned entries (Sigma A_l)           */
     int64_t arcs_walked;   /* arcs walked by the peel (= m for a full run)            */
     int64_t compactions;   /* alive-list rewrites                                      */
-    int64_t hub_arcs;      /* pool entries (<= 4096 arcs each) shared between CTAs     */
+    int64_t hub_arcs;      /* arcs walked in grid-wide (global queue) HUB phases       */
     int32_t kmax;          /* largest core number                                     */
     int32_t grid_blocks;   /* persistent grid size                                     */
     int32_t block_threads;
@@ -133,7 +133,7 @@ int kcore_decompose_host(const int64_t *rowptr_host, const int32_t *colidx_host,
                          const kcore_options *opt, kcore_stats *stats);
 
 /* Scratch bytes needed by kcore_decompose_ex for a graph with n vertices and
- * m arcs (about 40 n + 4 m / 1024 bytes + 64 KiB). */
+ * m arcs (about 36 n bytes + 4 KiB). */
 size_t kcore_workspace_size(int64_t n, int64_t m);
 
 /* Check the CSR preconditions on the device (DEVICE pointers): rowptr[0]==0,

@@ -1,46 +1,43 @@
-// kc_kernels.cuh -- sm_100a kernels of the k-core hot path (v5).
+// kc_kernels.cuh -- sm_100a kernels of the k-core hot path (v3).
 //
 // One call = one persistent cooperative kernel (k_persistent), one CTA per SM,
 // running the whole decomposition as a device-resident state machine.  Per
-// level k (Alg. 1's round) there is ONE grid phase and one grid
-// barrier:
+// level k (Alg. 1's round) there is ONE grid phase:
 //
-//   scan   every CTA scans its segment of the alive list (Alg. 2):
-//          deg[v] == k -> v is in the k-shell: claim it, append it to the
-//                         CTA's LOCAL frontier (shared memory) or, if it is
-//                         big or the frontier is full, to the global POOL;
-//          deg[v] >  k -> running min for the level skip; alive-list compaction.
-//   drain  the CTA drains its local frontier breadth-first with CTA-local
-//          sub-rounds (__syncthreads only) -- the paper's block-local BFS of
-//          Alg. 3.  For every arc (v,u) (Alg. 3 l.19-24):
-//            if deg[u] > k: old = atomicSub(&deg[u],1)
-//               old == k+1 -> u reached k: claim, append to the next local
-//                             frontier (or the pool)
-//               old <= k   -> atomicAdd(&deg[u],1)  (restore, Fig. 6)
-//               else       -> min_next = min(min_next, old-1)          (level skip)
-//   pool   vertices too big for a CTA-local sub-round, or overflowing it, go
-//          to a global pool (one packed atomic reserves entries and their
-//          range in the pool's ARC space).  A CTA with no local work claims a
-//          range of pool arcs (CAS, never past the reserved arcs) and walks it
-//          with all its warps, arc-balanced (hubs are shared by many CTAs),
-//          then drains the local frontier that produced -- asynchronous work
-//          sharing, no sub-round barrier.  The level ends when every CTA has
-//          finished its scan and the pool's done arcs equal its reserved arcs.
-//   level end: k <- max(k+1, min_next)  (Alg. 1 l.9 does k+1; reading R5)
+//   LEVEL(k)  every CTA scans its tiles of the alive list (Alg. 2):
+//             deg[v] == k  -> v is in the k-shell: claim it, append it to the
+//                             CTA's LOCAL frontier (shared memory);
+//             deg[v] >  k  -> running min for the level skip, optional
+//                             alive-list compaction;
+//             then drains its local frontier breadth-first with CTA-local
+//             sub-rounds (__syncthreads only) -- the paper's block-local BFS
+//             of Alg. 3.  For every arc (v,u) (Alg. 3 l.19-24):
+//               if deg[u] > k: old = atomicSub(&deg[u],1)
+//                  old == k+1 -> u reached k: claim it, append it to the next
+//                                local frontier
+//                  old <= k   -> atomicAdd(&deg[u],1)  (restore, Fig. 6)
+//                  else       -> min_next = min(min_next, old-1)    (level skip)
+//   HUB       vertices too big for one CTA (> kHub arcs) or overflowing a
+//             local frontier go to a global queue; a HUB phase splits that
+//             queue's ARCS evenly over every warp of the grid, then drains
+//             the resulting local frontiers the same way.
+//   level end k <- max(k+1, min_next)  (Alg. 1 l.9 does k+1; reading R5)
 //
-// Scans and drains of one level run concurrently in different CTAs, so a
-// vertex can be seen with deg == k by a scan and reached (old == k+1) by a
-// peel; a claim bit per vertex (atomicOr) makes removal exactly-once
-// (DESIGN.md reading R9).
+// Scan and drain run concurrently in different CTAs, so a vertex can be seen
+// with deg == k by a scan and reached (old == k+1) by a peel in the same
+// level; a claim bit per vertex (atomicOr) makes removal exactly-once
+// (DESIGN.md reading R9; SURVEY Q9).
 //
 // Control: every CTA keeps an identical copy of the control state in shared
 // memory; a phase ends with a grid barrier whose last arriver snapshots and
-// resets the counters, and every CTA applies the same pure advance().  Levels
-// over a short alive list run `solo` on CTA 0 with CTA-local sync only.
+// resets the counters, and every CTA applies the same pure advance().  Phases
+// over a short alive list / few arcs run `solo` on CTA 0 with CTA-local sync.
 //
-// Filter: a CTA that walks many arcs in a level whose alive list is short
-// builds a Bloom filter of that list in shared memory; arcs whose target is
-// definitely not alive skip the scattered deg[] read.
+// Filter: when a CTA has many arcs to walk and the alive list at level start
+// is short, it builds a Bloom filter of that list in shared memory; arcs whose
+// target is definitely not alive (removed at an earlier level) then skip the
+// scattered deg[] read entirely (the read is the throughput limiter, see
+// DESIGN.md "Measured primitives").
 #pragma once
 
 #include "kc_common.cuh"
@@ -51,63 +48,63 @@ namespace kc {
 constexpr int kBlock = 768;
 constexpr int kWarps = kBlock / 32;
 constexpr int kScanItems = 8;        // alive-list entries per lane per warp step
-constexpr int kLCap = kBlock;        // local frontier capacity (one entry per thread in the prefix)
-constexpr int kSub = 8192;           // arc budget of one CTA-local sub-round
-constexpr int kPStage = 64;          // per-warp pool stage (vertices)
-constexpr int kClaimMin = 4096;      // pool ARCS claimed at a time: backlog / (2 grid),
-constexpr int kClaimMax = 1 << 19;   //   clamped to [kClaimMin, kClaimMax]
-constexpr int kMaxLocalRounds = 4;   // then the local frontier goes back to the pool
-constexpr int kSoloBail = 16384;     // a solo level with more pending pool arcs goes grid-wide
+constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)
+// CTA-local routing budgets (arcs), chosen per level from the size of the
+// previous level: light levels keep their BFS local, heavy ones go grid-wide.
+constexpr int kLightLevelArcs = 4 << 20;
+constexpr int kHubLight = 32768, kSubLight = 32768, kPhaseLight = 262144;
+constexpr int kHubHeavy = 8192, kSubHeavy = 8192, kPhaseHeavy = 16384;
+constexpr int kGStage = 64;          // per-warp global-queue stage (any size; flushed 32 at a time)
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
 constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
-constexpr int kUnroll = 4;           // arcs per lane in flight per batch (handle_hits assumes 4)
+constexpr int kUnroll = 4;  // arcs per lane in flight per batch (handle_hits assumes 4)
 constexpr int kBatch = 32 * kUnroll;
 constexpr int kTraceFields = 8;
 
-enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_DONE = 3 };
+enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
 struct Ctrl {
     int32_t phase, solo, k, level_min;
     int32_t compact, src_sel, dst_sel, alive_sel;
     int32_t src_single, alive_single;  // 1: the list is one contiguous run in segment 0
-    int32_t cont;                      // 1: the level's scan is done, only the pool is left
+    int32_t light;                     // budgets of this level (see kLightLevelArcs)
     int32_t pad1;
+    int64_t arcs_lvl0;                 // arcs walked when the level began
+    int64_t pad2;
     int64_t src_len, alive_len;
-    int64_t scan_target;               // scans_done value that ends the current level
-    int64_t ord_lvl0;                  // removed count when the level began
-    int64_t level;                     // level index (for the Bloom cache)
-    int64_t st_levels, st_phases, st_solo, st_bar, st_scanned, st_compact, st_pool;
+    int64_t s, e, as, ae;          // HUB: global-queue slots [s,e), arcs [as,ae)
+    int64_t gq_cnt, gq_arc;        // global queue consumed so far
+    int64_t ord_lvl0;              // order tail when the level began
+    int64_t level;                 // level index (for the Bloom cache)
+    int64_t st_levels, st_phases, st_solo, st_bar, st_scanned, st_compact, st_hubarcs;
     int32_t st_kmax, st_pad;
-    int64_t alive_carry;               // compaction output already counted (solo bail-out)
 };
 
 static_assert(sizeof(Ctrl) % 16 == 0, "Ctrl is copied as int4");
 
 struct Snap {
-    unsigned long long ord;        // removed vertices
+    unsigned long long arcs;       // arcs walked so far
+    unsigned long long gq;         // packed global-queue tail
+    unsigned long long ord;        // order tail (= removed vertices)
     unsigned long long alive_out;  // compaction output length
-    unsigned long long pool;       // pool entries so far
     int32_t min;
     int32_t pad;
 };
 
 struct Params {
     int64_t n;
-    int32_t solo_arcs;  // unused (kept for the options ABI)
-    int32_t solo_scan;  // levels over <= this many alive entries run solo
+    int32_t solo_arcs;  // HUB phases with <= this many arcs run solo
+    int32_t solo_scan;  // LEVEL phases over <= this many entries run solo
     int32_t bloom;      // 0 disables the Bloom filter
     int32_t pad;
 };
 
 struct State {
-    alignas(128) unsigned long long ord_tail;   // removed vertices (order slots if recorded)
+    alignas(128) unsigned long long gq_tail;    // packed (count << 33) | arcs
+    alignas(128) unsigned long long ord_tail;   // vertices written to order[]
     alignas(128) unsigned long long alive_out;  // compaction output length
     alignas(128) int32_t min_next;              // atomicMin target
-    alignas(128) unsigned long long pool_tail;  // packed (entries << 33) | arcs reserved
-    alignas(128) unsigned long long pool_claim; // pool arcs claimed
-    alignas(128) unsigned long long pool_done;  // pool arcs fully processed
-    alignas(128) unsigned long long scans_done; // CTA scans finished (monotone)
     alignas(128) uint32_t bar_count;            // grid barrier arrivals (monotone)
     alignas(128) uint32_t bar_gen;              // grid barrier generation
     Snap snap[2];                               // counters at barrier gen, by gen & 1
@@ -123,15 +120,13 @@ struct State {
 struct KArgs {
     const int64_t *rowptr;
     const int32_t *colidx;
-    int32_t *deg;         // == core_out
-    int32_t *order;       // removal order, or nullptr when not requested
-    uint32_t *claimed;    // claim bit per vertex
-    int32_t *pool_v;      // pool entry j: vertex,
-    int64_t *pool_beg;    //   its first arc in colidx,
-    int64_t *pool_P;      //   its first arc in the pool's arc space (prefix),
-    int32_t *pool_len;    //   its arcs (0 = not yet published; zeroed at init)
-    int64_t pool_cap;
-    int32_t *alive[2];    // alive lists, one segment per CTA
+    int32_t *deg;       // == core_out
+    int32_t *order;     // removal order (all vertices)
+    uint32_t *claimed;  // claim bit per vertex
+    int32_t *gq_v;      // global queue: vertex, row begin, arc prefix
+    int64_t *gq_beg;
+    int64_t *gq_arc;
+    int32_t *alive[2];  // alive lists, partitioned into nseg per-CTA segments
     int32_t *seg_len[2];  // entries of segment b in alive[x]: seg_len[x][b]
     int64_t seg_R;        // segment region size: segment b lives at [b*R, b*R + len)
     int32_t nseg;         // = persistent grid size
@@ -147,22 +142,22 @@ struct Smem {
     int64_t lpre[kLCap + 1];
     int32_t lcnt[2];
     int32_t larc[2];
+    int32_t lphase;      // local arcs accepted this phase
     int32_t removed;     // vertices removed by this CTA this phase (order not recorded)
-    int32_t kcur;        // scan: compaction cursor
-    int32_t pv[kWarps][kPStage];
-    int32_t pd[kWarps][kPStage];
-    int64_t pb[kWarps][kPStage];
+    int32_t fit;         // unused
+    int32_t kcur;        // scan: compaction cursor within the current segment
+    int32_t bud_hub, bud_sub, bud_phase, bud_pad;  // routing budgets of this phase
+    unsigned long long scan_q2[kWarps];
+    unsigned long long tot_q2, base_g, base_w;
+    int32_t gv[kWarps][kGStage];
+    int32_t gd[kWarps][kGStage];
+    int64_t gb[kWarps][kGStage];
     unsigned long long scan_q[kWarps];
-    unsigned long long tot_q;
+    unsigned long long tot_q, base_o, base_k;
     int32_t red_min[kWarps];
-    int64_t c0, c1;      // claimed pool arcs
-    int64_t cnt;         // pool entries reserved when they were claimed
-    int64_t backlog;     // unclaimed pool arcs per CTA when they were claimed
-    int32_t done, pad3;
-    int64_t lvl_arcs;    // arcs this CTA walked in the current level
     int64_t bloom_level;
     int32_t bloom_on;
-    int32_t pad4;
+    int32_t pad;
     Ctrl ctrl;
     Snap snap;
     uint32_t bloom[kBloomWords];
@@ -176,25 +171,18 @@ __device__ __forceinline__ int warp_min(int v)
     return v;
 }
 
+__device__ __forceinline__ int64_t warp_sum64(int64_t v)
+{
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(kFull, v, o);
+    return v;
+}
+
 __device__ __forceinline__ unsigned long long globaltimer()
 {
     unsigned long long t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
-}
-
-__device__ __forceinline__ unsigned long long ld_acquire_u64(const unsigned long long *p)
-{
-    unsigned long long v;
-    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-
-__device__ __forceinline__ int32_t ld_acquire_i32(const int32_t *p)
-{
-    int32_t v;
-    asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
 }
 
 __device__ __forceinline__ uint32_t bloom_h1(uint32_t v) { return (v * 0x9E3779B1u) >> 12; }
@@ -206,9 +194,9 @@ __device__ __forceinline__ bool bloom_maybe(const Smem &sm, uint32_t v)
     return ((sm.bloom[a >> 5] >> (a & 31)) & (sm.bloom[b >> 5] >> (b & 31)) & 1u) != 0;
 }
 
-// Per-CTA timestamps of the current phase (trace mode only), indexed by the
-// number of grid barriers passed: 0 start, 1 end of own scan, 2 end of own
-// drain, 3 barrier arrival (after the pool loop).
+// Per-CTA timestamps of the current phase (trace mode only): slot 0 phase
+// start, 1 end of scan / queue walk, 2 end of local drain, 3 barrier arrival.
+// Indexed by the number of grid barriers passed (identical in every CTA).
 __device__ __forceinline__ void cta_time(const KArgs &A, const Ctrl &c, int slot)
 {
     if (threadIdx.x != 0 || c.solo) return;
@@ -259,75 +247,89 @@ __device__ __forceinline__ unsigned long long block_excl_scan(Smem &sm, unsigned
     return sm.scan_q[wib] + (qi - q);
 }
 
-__device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
+// Block-wide exclusive scans of two u64 per thread; totals in tot_q / tot_q2.
+__device__ __forceinline__ void block_excl_scan2(Smem &sm, unsigned long long q, unsigned long long r,
+                                                 unsigned long long &qe, unsigned long long &re)
 {
-    const uint32_t bit = 1u << (v & 31);
-    return (atomicOr(A.claimed + (v >> 5), bit) & bit) == 0u;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    unsigned long long qi = q, ri = r;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long t = __shfl_up_sync(kFull, qi, o);
+        const unsigned long long t2 = __shfl_up_sync(kFull, ri, o);
+        if (lane >= o) { qi += t; ri += t2; }
+    }
+    if (lane == 31) { sm.scan_q[wib] = qi; sm.scan_q2[wib] = ri; }
+    __syncthreads();
+    if (wib == 0) {
+        const unsigned long long wq = lane < kWarps ? sm.scan_q[lane] : 0ULL;
+        const unsigned long long wr = lane < kWarps ? sm.scan_q2[lane] : 0ULL;
+        unsigned long long iq = wq, ir = wr;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long t = __shfl_up_sync(kFull, iq, o);
+            const unsigned long long t2 = __shfl_up_sync(kFull, ir, o);
+            if (lane >= o) { iq += t; ir += t2; }
+        }
+        if (lane < kWarps) { sm.scan_q[lane] = iq - wq; sm.scan_q2[lane] = ir - wr; }
+        if (lane == kWarps - 1) { sm.tot_q = iq; sm.tot_q2 = ir; }
+    }
+    __syncthreads();
+    qe = sm.scan_q[wib] + (qi - q);
+    re = sm.scan_q2[wib] + (ri - r);
 }
 
-// ------------------------------------------------------------- the pool
-// Flush this warp's pool stage: one packed atomic reserves the entries and
-// their range in the pool's arc space; entries are published by writing their
-// length last, after a fence (consumers spin until it is non-zero).
-__device__ __noinline__ void pool_flush(const KArgs &A, Smem &sm, int wib, int &pcnt)
+// ------------------------------------------------------------ warp stages
+// Global queue: one packed atomic reserves slots and their arc range.
+__device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
-    if (pcnt == 0) return;
+    if (gcnt == 0) return;
     __syncwarp();
-    int64_t dd[2], pre[2];
-    int64_t carry = 0;
-#pragma unroll
-    for (int h = 0; h < 2; h++) {
-        const int x = h * 32 + lane;
-        dd[h] = x < pcnt ? (int64_t)sm.pd[wib][x] : 0;
-        int64_t incl = dd[h];
+    int64_t tot = 0;
+    for (int x = lane; x < gcnt; x += 32) tot += sm.gd[wib][x];
+    tot = warp_sum64(tot);
+    unsigned long long base = 0;
+    if (lane == 0)
+        base = atomicAdd(&A.S->gq_tail, ((unsigned long long)gcnt << kArcBits) | (unsigned long long)tot);
+    base = __shfl_sync(kFull, base, 0);
+    const int64_t bc = (int64_t)(base >> kArcBits);
+    int64_t carry = (int64_t)(base & kArcMask);
+    for (int x0 = 0; x0 < gcnt; x0 += 32) {
+        const int x = x0 + lane;
+        const int64_t d = x < gcnt ? (int64_t)sm.gd[wib][x] : 0;
+        int64_t incl = d;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             const int64_t t = __shfl_up_sync(kFull, incl, o);
             if (lane >= o) incl += t;
         }
-        pre[h] = carry + incl - dd[h];
+        if (x < gcnt) {
+            A.gq_v[bc + x] = sm.gv[wib][x];
+            A.gq_beg[bc + x] = sm.gb[wib][x];
+            A.gq_arc[bc + x] = carry + incl - d;
+        }
         carry += __shfl_sync(kFull, incl, 31);
     }
-    unsigned long long base = 0;
-    if (lane == 0)
-        base = atomicAdd(&A.S->pool_tail, ((unsigned long long)pcnt << kArcBits) | (unsigned long long)carry);
-    base = __shfl_sync(kFull, base, 0);
-    const int64_t bc = (int64_t)(base >> kArcBits), ba = (int64_t)(base & kArcMask);
-#pragma unroll
-    for (int h = 0; h < 2; h++) {
-        const int x = h * 32 + lane;
-        if (x < pcnt) {
-            A.pool_v[bc + x] = sm.pv[wib][x];
-            A.pool_beg[bc + x] = sm.pb[wib][x];
-            A.pool_P[bc + x] = ba + pre[h];
-        }
-    }
-    __threadfence();
-#pragma unroll
-    for (int h = 0; h < 2; h++) {
-        const int x = h * 32 + lane;
-        if (x < pcnt) A.pool_len[bc + x] = (int32_t)dd[h];
-    }
     __syncwarp();
-    pcnt = 0;
+    gcnt = 0;
 }
 
-// Route claimed vertices (one per lane where `won`): record the removal
-// (order slot if requested -- a vertex is claimed only after every vertex
+// Route claimed vertices (one per lane where `won`): reserve their slots in
+// the removal order right away (a vertex is claimed only after every vertex
 // whose processing made it reach k was claimed, so claim-time slots form a
-// valid peel order, the I4 certificate -- else a count), then send each to
-// the local next frontier `nx` if it fits the sub-round's arc budget, else
-// to the pool.  Zero-degree vertices are only recorded.
-__device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool won, int32_t v,
-                                          int32_t dv, int64_t bv, int nx, int &pcnt)
+// valid peel order -- the I4 certificate), then send each to the local next
+// frontier `nx` if it is small and fits the sub-round's arc budget, else to
+// the global queue.  Zero-degree vertices are only recorded.
+__device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool won, int32_t v,
+                                          int32_t dv, int64_t bv, int nx, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
     const unsigned b = __ballot_sync(kFull, won);
     if (b == 0) return;
     {
         const int lead = __ffs(b) - 1;
-        if (A.order) {
+        if (A.order) {  // peel order requested: slots in claim order
             unsigned long long base = 0;
             if (lane == lead) base = atomicAdd(&A.S->ord_tail, (unsigned long long)__popc(b));
             base = __shfl_sync(kFull, base, lead);
@@ -336,7 +338,7 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
             atomicAdd(&sm.removed, __popc(b));
         }
     }
-    const bool cand = won && dv > 0 && dv <= kSub;
+    const bool cand = won && dv > 0 && dv <= sm.bud_hub;
     const unsigned bc = __ballot_sync(kFull, cand);
     bool wantl = false;
     int lbase = 0;
@@ -345,16 +347,20 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) sumd += __shfl_xor_sync(kFull, sumd, o);
         const int lead = __ffs(bc) - 1;
+        int oa = 0;
         int ok = 0;
         if (lane == lead) {
-            const int oa = atomicAdd(&sm.larc[nx], sumd);
-            if (oa + sumd <= kSub) { ok = 1; lbase = atomicAdd(&sm.lcnt[nx], __popc(bc)); }
+            oa = atomicAdd(&sm.larc[nx], sumd);
+            if (oa + sumd <= sm.bud_sub) {
+                const int op = atomicAdd(&sm.lphase, sumd);
+                if (op + sumd <= sm.bud_phase) { ok = 1; lbase = atomicAdd(&sm.lcnt[nx], __popc(bc)); }
+            }
         }
         ok = __shfl_sync(kFull, ok, lead);
         lbase = __shfl_sync(kFull, lbase, lead);
         wantl = cand && ok;
     }
-    bool top = won && dv > 0 && !wantl;
+    bool tog = won && dv > 0 && !wantl;
     if (wantl) {
         const int pos = lbase + __popc(bc & lanemask_lt());
         if (pos < kLCap) {
@@ -362,29 +368,35 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
             sm.ld[nx][pos] = dv;
             sm.lb[nx][pos] = bv;
         } else {
-            top = true;
+            tog = true;
         }
     }
-    const unsigned bg = __ballot_sync(kFull, top);
+    const unsigned bg = __ballot_sync(kFull, tog);
     if (bg) {
         const int c = __popc(bg);
-        if (pcnt + c > kPStage) pool_flush(A, sm, wib, pcnt);
-        if (top) {
-            const int pos = pcnt + __popc(bg & lanemask_lt());
-            sm.pv[wib][pos] = v;
-            sm.pd[wib][pos] = dv;
-            sm.pb[wib][pos] = bv;
+        if (gcnt + c > kGStage) gq_flush(A, sm, wib, gcnt);
+        if (tog) {
+            const int pos = gcnt + __popc(bg & lanemask_lt());
+            sm.gv[wib][pos] = v;
+            sm.gd[wib][pos] = dv;
+            sm.gb[wib][pos] = bv;
         }
-        pcnt += c;
+        gcnt += c;
     }
     __syncwarp();
+}
+
+__device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
+{
+    const uint32_t bit = 1u << (v & 31);
+    return (atomicOr(A.claimed + (v >> 5), bit) & bit) == 0u;
 }
 
 // --------------------------------------------------------- arc walking
 // Hits of one batch (u reached k): claim, fetch row bounds, prefetch the
 // row's first line for the next hop, route.  Out of line: rare path.
 __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u0, int u1, int u2, int u3,
-                                         unsigned hm, int &pcnt)
+                                         unsigned hm, int &gcnt)
 {
     const int wib = threadIdx.x >> 5;
     const int uu[4] = {u0, u1, u2, u3};
@@ -400,26 +412,32 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u
 #pragma unroll
     for (int r = 0; r < 4; r++) {
         if (won[r] && b1[r] > b0[r]) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[r]));
-        route_won(A, sm, wib, won[r], uu[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, pcnt);
+        route_won(A, sm, wib, won[r], uu[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, gcnt);
     }
 }
 
-// Walk arcs [a0,a1) of the local frontier `cur` (entries [0,e), arc prefix
-// lpre[], row begins lb[cur][]; the last entry ends at arc ae) with one warp.
-// Each lane holds one entry of a 32-entry window; an arc finds its entry with
-// a 5-step shuffle search on 32-bit offsets relative to the current batch.
+// Walk arcs [a0,a1) of a frontier whose entries are i = [s,e) with arc
+// prefix P(i) and row begin B(i); the last entry ends at arc ae.  LOCAL=true:
+// entries live in this CTA's shared-memory list `cur`; else in the global
+// queue.  Hits are routed into local list `nx`.  Each lane holds one entry
+// of a 32-entry window; an arc finds its entry with a 5-step shuffle search
+// on 32-bit offsets relative to the current batch.
+template <bool LOCAL>
 __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, const int cur, const int nx,
-                                     int64_t e, int64_t ae, int64_t a0, int64_t a1, bool use_bloom,
-                                     int &lmin, int &pcnt)
+                                     int64_t s, int64_t e, int64_t ae, int64_t a0, int64_t a1,
+                                     bool use_bloom, int &lmin, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
-    int64_t lo = 0, hi = e;  // first entry: largest i with lpre[i] <= a0 (32-ary search)
+    // first entry: largest i in [s,e) with P(i) <= a0 (32-ary search)
+    int64_t lo = s, hi = e;
     while (true) {
         const int64_t step = hi - lo > 32 ? (hi - lo + 31) / 32 : 1;
         const int64_t p = lo + lane * step;
-        const bool ok = (p < hi) && sm.lpre[p] <= a0;
+        bool ok = false;
+        if (p < hi) ok = (LOCAL ? sm.lpre[p] : ld_cg_i64(A.gq_arc + p)) <= a0;
         const unsigned b = __ballot_sync(kFull, ok);
-        lo = lo + (31 - __clz(b)) * step;
+        const int L = 31 - __clz(b);
+        lo = lo + L * step;
         if (step == 1) break;
         hi = min(hi, lo + step);
     }
@@ -429,15 +447,16 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
         const int64_t j = i + lane;
         int64_t wq = LLONG_MAX, wbeg = 0;
         if (j < e) {
-            wq = sm.lpre[j];
-            wbeg = sm.lb[cur][j];
+            wq = LOCAL ? sm.lpre[j] : ld_cg_i64(A.gq_arc + j);
+            wbeg = LOCAL ? sm.lb[cur][j] : ld_cg_i64(A.gq_beg + j);
         }
         int64_t nxt = __shfl_down_sync(kFull, wq, 1);
         if (j + 1 >= e) nxt = ae;
-        else if (lane == 31) nxt = sm.lpre[j + 1];
+        else if (lane == 31) nxt = LOCAL ? sm.lpre[j + 1] : ld_cg_i64(A.gq_arc + j + 1);
         const int64_t limit = min(a1, __shfl_sync(kFull, nxt, 31));
         const int64_t bmq = wbeg - wq;  // colidx index of arc x in this entry = bmq + x
         while (a < limit) {
+            // window starts relative to this batch, clamped to int32
             const int64_t rq = wq - a;
             const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
             const int32_t lim = (int32_t)min((int64_t)kBatch, limit - a);
@@ -472,7 +491,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
                 else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
                 else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
             }
-            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, pcnt);
+            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, gcnt);
             a += kBatch;
         }
         a = limit;
@@ -480,91 +499,35 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
     }
 }
 
-// Pool entry j (spinning until it is published): arc-space start, length, row begin.
-__device__ __forceinline__ int32_t pool_entry(const KArgs &A, int64_t j, int64_t &P, int64_t &beg)
+// Drain this CTA's local frontier (list `cur`) breadth-first with CTA-local
+// sub-rounds.  Returns the number of arcs walked.
+__device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, bool use_bloom,
+                               int &lmin, int &gcnt)
 {
-    int32_t len;
-    while ((len = ld_acquire_i32(A.pool_len + j)) == 0) {
-    }
-    P = ld_cg_i64(A.pool_P + j);
-    beg = ld_cg_i64(A.pool_beg + j);
-    return len;
-}
-
-// Walk pool arcs [a0,a1) with one warp (entries [0,cnt) are reserved; every
-// arc below a1 belongs to one of them).  Same window scheme as walk().
-__device__ __forceinline__ void walk_pool(const KArgs &A, Smem &sm, const int k, const int nx, int64_t cnt,
-                                          int64_t a0, int64_t a1, bool use_bloom, int &lmin, int &pcnt)
-{
-    const int lane = threadIdx.x & 31;
-    int64_t lo = 0, hi = cnt;  // first entry: largest j with P(j) <= a0
+    const int wib = threadIdx.x >> 5;
+    int64_t walked = 0;
     while (true) {
-        const int64_t step = hi - lo > 32 ? (hi - lo + 31) / 32 : 1;
-        const int64_t p = lo + lane * step;
-        bool ok = false;
-        if (p < hi) {
-            int64_t P, beg;
-            pool_entry(A, p, P, beg);
-            ok = P <= a0;
-        }
-        const unsigned b = __ballot_sync(kFull, ok);
-        lo = lo + (31 - __clz(b)) * step;
-        if (step == 1) break;
-        hi = min(hi, lo + step);
+        __syncthreads();
+        const int L = min(sm.lcnt[cur], kLCap);
+        if (L == 0) break;
+        // arc prefix of the list
+        const int64_t dv = threadIdx.x < L ? (int64_t)sm.ld[cur][threadIdx.x] : 0;
+        const unsigned long long ex = block_excl_scan(sm, (unsigned long long)dv);
+        if (threadIdx.x < L) sm.lpre[threadIdx.x] = (int64_t)ex;
+        const int64_t T = (int64_t)sm.tot_q;
+        const int nx = cur ^ 1;
+        if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; sm.larc[nx] = 0; }
+        __syncthreads();
+        int64_t C = (T + kWarps - 1) / kWarps;
+        C = ((C + kBatch - 1) / kBatch) * kBatch;
+        const int64_t a0 = (int64_t)wib * C;
+        if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, lmin, gcnt);
+        walked += T;
+        __syncthreads();
+        if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
+        cur = nx;
     }
-    int64_t i = lo;
-    int64_t a = a0;
-    while (a < a1) {
-        const int64_t j = i + lane;
-        int64_t wq = LLONG_MAX, wbeg = 0, wend = LLONG_MAX;
-        if (j < cnt) {
-            const int32_t len = pool_entry(A, j, wq, wbeg);
-            wend = wq + len;
-        }
-        const int last = (int)min((int64_t)31, cnt - 1 - i);
-        const int64_t limit = min(a1, __shfl_sync(kFull, wend, last));
-        const int64_t bmq = wbeg - wq;
-        while (a < limit) {
-            const int64_t rq = wq - a;
-            const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
-            const int32_t lim = (int32_t)min((int64_t)kBatch, limit - a);
-            int32_t u[kUnroll];
-#pragma unroll
-            for (int r = 0; r < kUnroll; r++) {
-                const int32_t my = r * 32 + lane;
-                int pos = 0;
-#pragma unroll
-                for (int bs = 16; bs >= 1; bs >>= 1) {
-                    const int32_t q = __shfl_sync(kFull, q32, pos + bs);
-                    if (q <= my) pos += bs;
-                }
-                const int64_t off = __shfl_sync(kFull, bmq, pos);
-                u[r] = (my < lim) ? ld_stream_i32(A.colidx + off + a + my) : -1;
-            }
-            if (use_bloom) {
-#pragma unroll
-                for (int r = 0; r < kUnroll; r++)
-                    if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
-            }
-            int32_t d[kUnroll];
-#pragma unroll
-            for (int r = 0; r < kUnroll; r++) d[r] = u[r] >= 0 ? ld_cg_i32(A.deg + u[r]) : -1;
-            int old[kUnroll];
-#pragma unroll
-            for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
-            unsigned hm = 0;
-#pragma unroll
-            for (int r = 0; r < kUnroll; r++) {
-                if (old[r] == k + 1) hm |= 1u << r;
-                else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
-                else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
-            }
-            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, pcnt);
-            a += kBatch;
-        }
-        a = limit;
-        i += 32;
-    }
+    return walked;
 }
 
 // Bloom filter of the alive list at level start (built once per level).
@@ -598,66 +561,14 @@ __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
     __syncthreads();
 }
 
-// Decide (CTA-uniform) whether the arcs this CTA walks this level pay for a filter.
-__device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &sm, int64_t more)
+// Decide (CTA-uniform) whether walking `arcs` arcs this phase pays for a filter.
+__device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &sm, int64_t arcs)
 {
     if (!A.S->prm.bloom || c.src_sel < 0 || c.src_len > kBloomMaxA) return false;
     if (sm.bloom_on && sm.bloom_level == c.level) return true;
-    if (sm.lvl_arcs + more < 4 * c.src_len + 65536) return false;
+    if (arcs < 4 * c.src_len + 65536) return false;
     bloom_build(A, c, sm);
     return true;
-}
-
-// Drain this CTA's local frontier (list `cur`) breadth-first with CTA-local
-// sub-rounds.  Returns the number of arcs walked.
-__device__ int64_t local_drain(const KArgs &A, const Ctrl &c, Smem &sm, int cur, int &lmin, int &pcnt)
-{
-    const int wib = threadIdx.x >> 5;
-    int64_t walked = 0;
-    for (int round = 0;; round++) {
-        __syncthreads();
-        const int L = min(sm.lcnt[cur], kLCap);
-        if (L == 0) break;
-        if (round == kMaxLocalRounds) {
-            // a long local chain: hand the frontier back to the pool so idle
-            // CTAs share it (each warp pushes a slice through its stage)
-            for (int x0 = wib * 32; x0 < L; x0 += kWarps * 32) {
-                const int x = x0 + (threadIdx.x & 31);
-                const bool has = x < L;
-                const unsigned bg = __ballot_sync(kFull, has);
-                if (pcnt + __popc(bg) > kPStage) pool_flush(A, sm, wib, pcnt);
-                if (has) {
-                    const int pos = pcnt + __popc(bg & lanemask_lt());
-                    sm.pv[wib][pos] = sm.lv[cur][x];
-                    sm.pd[wib][pos] = sm.ld[cur][x];
-                    sm.pb[wib][pos] = sm.lb[cur][x];
-                }
-                pcnt += __popc(bg);
-                __syncwarp();
-            }
-            __syncthreads();
-            if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
-            __syncthreads();
-            break;
-        }
-        const int64_t dv = threadIdx.x < L ? (int64_t)sm.ld[cur][threadIdx.x] : 0;
-        const unsigned long long ex = block_excl_scan(sm, (unsigned long long)dv);
-        if (threadIdx.x < L) sm.lpre[threadIdx.x] = (int64_t)ex;
-        const int64_t T = (int64_t)sm.tot_q;
-        const int nx = cur ^ 1;
-        if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; sm.larc[nx] = 0; }
-        __syncthreads();
-        const bool bl = want_bloom(A, c, sm, T);
-        int64_t C = (T + kWarps - 1) / kWarps;
-        C = ((C + kBatch - 1) / kBatch) * kBatch;
-        const int64_t a0 = (int64_t)wib * C;
-        if (a0 < T) walk(A, sm, c.k, cur, nx, L, T, a0, min(a0 + C, T), bl, lmin, pcnt);
-        walked += T;
-        __syncthreads();
-        if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; sm.lvl_arcs += T; }
-        cur = nx;
-    }
-    return walked;
 }
 
 // ------------------------------------------------------------------ INIT
@@ -672,21 +583,18 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
         lmin = min(lmin, d);
     }
     for (int64_t w = tid; w < (A.n + 31) / 32; w += stride) A.claimed[w] = 0u;
-    for (int64_t w = tid; w < A.pool_cap; w += stride) A.pool_len[w] = 0;
-    if (threadIdx.x == 0) {
-        sm.bloom_on = 0; sm.bloom_level = -1;
-        sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
-    }
+    if (threadIdx.x == 0) { sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
 // ------------------------------------------------------------------ LEVEL
-// Scan entries [lo,hi) of list `src` (nullptr: the identity) with every warp
-// of this CTA (Alg. 2): eight entries per lane in flight; deg == k -> claim +
-// route; deg > k -> min and ballot compaction (Fig. 8(c)) into dst[0..) with a
-// shared-memory cursor.  No block sync, no global atomics.
+// Scan entries [lo,hi) of list `src` (nullptr: the identity, ids lo..hi-1)
+// with every warp of this CTA (Alg. 2): eight entries per lane in flight;
+// deg == k -> claim + route (local frontier or global queue); deg > k ->
+// min for the level skip and, when compacting, ballot compaction (Fig. 8(c))
+// into dst[0..) with a shared-memory cursor.  No block sync, no global atomics.
 __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_t *src, int64_t lo,
-                           int64_t hi, int32_t *dst, int &lmin, int &pcnt)
+                           int64_t hi, int32_t *dst, int &lmin, int &gcnt)
 {
     const int k = c.k;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -709,8 +617,7 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
             else if (dd[j] > k) { lmin = min(lmin, dd[j]); km |= 1u << j; }
         }
         if (dst) {
-            const int mine = __popc(km);
-            int incl = mine;
+            int mine = __popc(km), incl = mine;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
                 const int t = __shfl_up_sync(kFull, incl, o);
@@ -725,6 +632,7 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
                 if ((km >> j) & 1u) dst[pos++] = vv[j];
         }
         if (__any_sync(kFull, wm != 0)) {
+            // row bounds of every claimed vertex first (all loads in flight), then route
             int64_t b0[kScanItems];
             int32_t du[kScanItems];
 #pragma unroll
@@ -738,7 +646,7 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
 #pragma unroll
             for (int j = 0; j < kScanItems; j++) {
                 if (du[j] > 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[j]));
-                route_won(A, sm, wib, (wm >> j) & 1u, vv[j], du[j], b0[j], 0, pcnt);
+                route_won(A, sm, wib, (wm >> j) & 1u, vv[j], du[j], b0[j], 0, gcnt);
             }
         }
     }
@@ -746,9 +654,10 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
 
 // Source layout: identity (src_sel < 0), one contiguous run (src_single) or
 // per-CTA segments.  Grid mode: CTA b scans its share and compacts into its
-// own segment b.  Solo mode: CTA 0 scans everything into one run (segment 0).
+// own segment b.  Solo mode: CTA 0 scans everything and compacts into one
+// contiguous run (segment 0).
 __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk, int &lmin,
-                           int &pcnt)
+                           int &gcnt)
 {
     const bool solo = (nblk == 1);
     const int32_t *srcb = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
@@ -758,16 +667,17 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
     __syncthreads();
     int32_t *dst = dstb ? dstb + (int64_t)dseg * A.seg_R : nullptr;
     if (c.src_sel < 0 || c.src_single) {
+        // contiguous source of c.src_len entries: an even slice per CTA
         const int64_t L = c.src_len;
         const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
-        scan_range(A, c, sm, srcb, lo, hi, dst, lmin, pcnt);
+        scan_range(A, c, sm, srcb, lo, hi, dst, lmin, gcnt);
     } else if (!solo) {
         const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + bid);
-        scan_range(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, pcnt);
+        scan_range(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt);
     } else {
         for (int b = 0; b < A.nseg; b++) {
             const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
-            if (len) scan_range(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, pcnt);
+            if (len) scan_range(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, gcnt);
         }
     }
     __syncthreads();
@@ -777,131 +687,114 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
     }
 }
 
-// One level (Alg. 1 round k): scan, drain the local frontier, then share the
-// pool until every CTA has scanned and every pool entry is processed.
-// c.cont: the scan was done by a solo CTA that bailed out; only the pool is
-// left.  A solo CTA (nblk == 1) bails out when its pool backlog is large and
-// returns true (the grid then finishes the level).
-__device__ bool phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+// One level (Alg. 1 round k): scan this CTA's segment(s), then drain the
+// local frontier breadth-first.
+__device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
 {
     const int wib = threadIdx.x >> 5;
-    State *S = A.S;
-    int lmin = INT_MAX, pcnt = 0;
-    int64_t walked = 0;
+    int lmin = INT_MAX, gcnt = 0;
     cta_time(A, c, 0);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
-        sm.removed = 0; sm.lvl_arcs = 0;
+        sm.lphase = 0; sm.removed = 0; sm.fit = 0;
+        sm.bud_hub = c.light ? kHubLight : kHubHeavy;
+        sm.bud_sub = c.light ? kSubLight : kSubHeavy;
+        sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
     }
     __syncthreads();
-    if (!c.cont) {
-        level_scan(A, c, sm, bid, nblk, lmin, pcnt);
-        cta_time(A, c, 1);
-        walked = local_drain(A, c, sm, 0, lmin, pcnt);
-        pool_flush(A, sm, wib, pcnt);
-        __syncthreads();
-    }
+    level_scan(A, c, sm, bid, nblk, lmin, gcnt);
+    __syncthreads();
+    cta_time(A, c, 1);
+    const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
+    const int64_t walked = local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
     cta_time(A, c, 2);
+    gq_flush(A, sm, wib, gcnt);
+    __syncthreads();
     if (threadIdx.x == 0) {
-        __threadfence();
-        atomicAdd(&S->scans_done, 1ULL);
-        sm.done = 0;
-        if (nblk == 1) {
-            const unsigned long long pend = (ld_acquire_u64(&S->pool_tail) & kArcMask) - ld_acquire_u64(&S->pool_done);
-            if (pend > (unsigned long long)kSoloBail) sm.done = 2;
-        }
+        if (walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+        if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
+    }
+    block_min_atomic(sm, lmin, &A.S->min_next);
+}
+
+// -------------------------------------------------------------------- HUB
+__device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+{
+    const int wib = threadIdx.x >> 5;
+    const int64_t gw = (int64_t)bid * kWarps + wib;
+    const int64_t W = (int64_t)nblk * kWarps;
+    const int64_t T = c.ae - c.as;
+    int64_t C = (T + W - 1) / W;
+    C = ((C + kBatch - 1) / kBatch) * kBatch;
+    int lmin = INT_MAX, gcnt = 0;
+    cta_time(A, c, 0);
+    if (threadIdx.x == 0) {
+        sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
+        sm.lphase = 0; sm.removed = 0; sm.fit = 0;
+        sm.bud_hub = c.light ? kHubLight : kHubHeavy;
+        sm.bud_sub = c.light ? kSubLight : kSubHeavy;
+        sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
     }
     __syncthreads();
-    const bool bail = sm.done == 2;
-    // pool loop: claim, copy into the local frontier, drain, report
-    bool bailed = bail;
-    while (!bailed) {
-        if (threadIdx.x == 0) {
-            int64_t c0 = -1, c1 = -1;
-            int done = 0;
-            const unsigned long long tp = ld_acquire_u64(&S->pool_tail);
-            const unsigned long long tcnt = tp >> kArcBits, tarc = tp & kArcMask;
-            unsigned long long cl = ld_acquire_u64(&S->pool_claim);
-            if (nblk == 1 && tarc - cl > (unsigned long long)kSoloBail) { cl = tarc; done = 2; }
-            while (cl < tarc) {
-                unsigned long long J = (tarc - cl) / (2ULL * (unsigned long long)nblk);
-                J = J < (unsigned long long)kClaimMin ? (unsigned long long)kClaimMin
-                                                      : (J > (unsigned long long)kClaimMax ? (unsigned long long)kClaimMax : J);
-                const unsigned long long want = min(cl + J, tarc);
-                const unsigned long long got = atomicCAS(&S->pool_claim, cl, want);
-                if (got == cl) { c0 = (int64_t)cl; c1 = (int64_t)want; break; }
-                cl = got;
-            }
-            if (c0 < 0 && done == 0) {
-                const unsigned long long dn = ld_acquire_u64(&S->pool_done);
-                const unsigned long long sd = ld_acquire_u64(&S->scans_done);
-                const unsigned long long t2 = ld_acquire_u64(&S->pool_tail) & kArcMask;
-                if (sd >= (unsigned long long)c.scan_target && dn == t2) done = 1;
-                else __nanosleep(64);
-            }
-            sm.c0 = c0;
-            sm.c1 = c1;
-            sm.cnt = (int64_t)tcnt;
-            sm.backlog = (int64_t)(tarc - (c0 < 0 ? tarc : (unsigned long long)c0)) / nblk;
-            sm.done = done;
-        }
-        __syncthreads();
-        if (sm.done == 2) { bailed = true; break; }
-        if (sm.done) break;
-        const int64_t c0 = sm.c0, c1 = sm.c1;
-        if (c0 < 0) continue;
-        // arc-balanced walk of the claimed pool arcs; hits go to local list 0
-        {
-            const int64_t T = c1 - c0;
-            const bool bl = want_bloom(A, c, sm, max(T, sm.backlog));
-            int64_t C = (T + kWarps - 1) / kWarps;
-            C = ((C + kBatch - 1) / kBatch) * kBatch;
-            const int64_t w0 = c0 + (int64_t)wib * C;
-            if (w0 < c1) walk_pool(A, sm, c.k, 0, sm.cnt, w0, min(w0 + C, c1), bl, lmin, pcnt);
-            walked += T;
-            __syncthreads();
-            if (threadIdx.x == 0) sm.lvl_arcs += T;
-        }
-        walked += local_drain(A, c, sm, 0, lmin, pcnt);  // starts with __syncthreads
-        pool_flush(A, sm, wib, pcnt);
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            __threadfence();
-            atomicAdd(&S->pool_done, (unsigned long long)(c1 - c0));
-        }
-    }
+    const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
+    const bool bl = want_bloom(A, c, sm, cta_arcs);
+    const int64_t a0 = c.as + gw * C;
+    if (a0 < c.ae)
+        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, lmin, gcnt);
+    int64_t walked = cta_arcs;
+    __syncthreads();
+    cta_time(A, c, 1);
+    walked += local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
+    cta_time(A, c, 2);
+    gq_flush(A, sm, wib, gcnt);
+    __syncthreads();
     if (threadIdx.x == 0) {
-        if (walked) atomicAdd(&S->arcs_walked, (unsigned long long)walked);
-        if (sm.removed) atomicAdd(&S->ord_tail, (unsigned long long)sm.removed);
+        if (walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+        if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
     }
-    block_min_atomic(sm, lmin, &S->min_next);
-    return bailed;
+    block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
 // ---------------------------------------------------------------- control
 // The pure transition function (Alg. 1 l.5-9 and the level skip).  Every CTA
 // applies it to identical inputs, so all copies stay identical.
-__device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p, int nblk)
+__device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
 {
+    const int64_t gcnt = (int64_t)(sn.gq >> kArcBits), garc = (int64_t)(sn.gq & kArcMask);
     const int64_t removed = (int64_t)sn.ord;
     c.level_min = min(c.level_min, sn.min);
     int next_k = 0;
+    bool new_level = false;
     if (c.phase == PH_INIT) {
         next_k = (c.level_min == INT_MAX) ? 0 : c.level_min;
         c.level_min = INT_MAX;
         c.level = -1;
-    } else {  // a LEVEL phase ended: the level is complete
+        new_level = true;
+    } else {
         c.st_phases++;
         if (c.solo) c.st_solo++;
-        c.st_scanned += c.src_len;
-        c.st_pool = (int64_t)sn.pool;
-        if (c.compact) {
-            c.alive_sel = c.dst_sel;
-            c.alive_len = (int64_t)sn.alive_out + c.alive_carry;
-            c.alive_single = c.solo || c.cont;  // a solo scan compacts into one run
-            c.st_compact++;
+        if (c.phase == PH_LEVEL) {
+            c.st_scanned += c.src_len;
+            if (c.compact) {
+                c.alive_sel = c.dst_sel;
+                c.alive_len = (int64_t)sn.alive_out;
+                c.alive_single = c.solo;  // a solo scan compacts into one run
+                c.st_compact++;
+            }
+        } else {
+            c.st_hubarcs += c.ae - c.as;
         }
+        if (gcnt > c.gq_cnt) {  // hub / overflow vertices pending: HUB phase
+            c.phase = PH_HUB;
+            c.s = c.gq_cnt; c.e = gcnt; c.as = c.gq_arc; c.ae = garc;
+            c.gq_cnt = gcnt; c.gq_arc = garc;
+            c.solo = (c.ae - c.as) <= (int64_t)p.solo_arcs;
+            return;
+        }
+        // level end
         if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
+        c.light = 0;  // adaptive budgets disabled: misjudge level jumps
+        (void)kLightLevelArcs;
         if (removed >= p.n) {
             c.phase = PH_DONE;
             c.solo = 0;
@@ -909,33 +802,36 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p, i
         }
         next_k = max(c.k + 1, c.level_min);
         c.level_min = INT_MAX;
+        new_level = true;
     }
-    const int64_t live = p.n - removed;
-    const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
-    c.phase = PH_LEVEL;
-    c.cont = 0;
-    c.alive_carry = 0;
-    c.k = next_k;
-    c.level++;
-    c.src_sel = c.alive_sel;
-    c.src_single = c.alive_single;
-    c.src_len = src_len;
-    c.compact = (live * 8 < src_len * 7) ? 1 : 0;  // >= 1/8 of the scan source is dead
-    c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
-    c.solo = src_len <= (int64_t)p.solo_scan;
-    // a solo scan of a segmented list gathers it into one run for next time
-    if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
-    c.scan_target += c.solo ? 1 : nblk;
-    c.ord_lvl0 = removed;
+    if (new_level) {
+        const int64_t live = p.n - removed;
+        const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
+        const bool compact = live * 8 < src_len * 7;  // >= 1/8 of the scan source is dead
+        c.phase = PH_LEVEL;
+        c.k = next_k;
+        c.level++;
+        c.src_sel = c.alive_sel;
+        c.src_single = c.alive_single;
+        c.src_len = src_len;
+        c.compact = compact ? 1 : 0;
+        c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
+        c.solo = src_len <= (int64_t)p.solo_scan;
+        // a solo scan of a segmented list gathers it into one run for next time
+        if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
+        c.ord_lvl0 = removed;
+        c.arcs_lvl0 = (int64_t)sn.arcs;
+    }
 }
 
 // Snapshot + reset of the counters (caller guarantees nobody else touches them).
 __device__ __forceinline__ Snap take_snapshot(State *S)
 {
     Snap sn;
+    sn.arcs = ld_relaxed_u64(&S->arcs_walked);
+    sn.gq = ld_relaxed_u64(&S->gq_tail);
     sn.ord = ld_relaxed_u64(&S->ord_tail);
     sn.alive_out = ld_relaxed_u64(&S->alive_out);
-    sn.pool = ld_relaxed_u64(&S->pool_tail) & kArcMask;
     sn.min = ld_relaxed_i32(&S->min_next);
     sn.pad = 0;
     S->alive_out = 0ULL;
@@ -943,7 +839,7 @@ __device__ __forceinline__ Snap take_snapshot(State *S)
     return sn;
 }
 
-__device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &sn, int grid, int64_t arcs)
+__device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &sn, int grid)
 {
     if (!S->trace) return;
     const unsigned long long i = S->trace_n;
@@ -953,8 +849,8 @@ __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &s
     r[1] = (int64_t)clock64();
     r[2] = ((int64_t)c.phase << 8) | ((int64_t)c.solo << 4) | grid;  // phase that ENDED
     r[3] = c.k;
-    r[4] = c.src_len;
-    r[5] = arcs;                  // arcs walked so far (cumulative)
+    r[4] = c.phase == PH_LEVEL ? c.src_len : (c.e - c.s);
+    r[5] = c.phase == PH_HUB ? (c.ae - c.as) : 0;
     r[6] = (int64_t)sn.ord;
     r[7] = c.st_bar;
     S->trace_n = i + 1;
@@ -979,9 +875,10 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
             while (ld_acquire_u32(&S->bar_gen) == gen) {
             }
             const Snap *ps = &S->snap[(gen + 1u) & 1u];
+            sn.arcs = ld_relaxed_u64(&ps->arcs);
+            sn.gq = ld_relaxed_u64(&ps->gq);
             sn.ord = ld_relaxed_u64(&ps->ord);
             sn.alive_out = ld_relaxed_u64(&ps->alive_out);
-            sn.pool = ld_relaxed_u64(&ps->pool);
             sn.min = ld_relaxed_i32(&ps->min);
             sn.pad = 0;
         }
@@ -990,33 +887,24 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
     __syncthreads();
 }
 
-// CTA 0 alone: run consecutive solo levels with CTA-local synchronisation.
+__device__ __forceinline__ void run_phase(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+{
+    if (c.phase == PH_LEVEL) phase_level(A, c, sm, bid, nblk);
+    else if (c.phase == PH_HUB) phase_hub(A, c, sm, bid, nblk);
+}
+
+// CTA 0 alone: run consecutive solo phases with CTA-local synchronisation.
 __device__ void solo_run(const KArgs &A, Smem &sm, const Params &p)
 {
     State *S = A.S;
     while (true) {
         const Ctrl c = sm.ctrl;
-        const bool bail = phase_level(A, c, sm, 0, 1);  // ends with __syncthreads
-        if (bail) {  // the level's pool is too big for one CTA: the grid finishes it
-            if (threadIdx.x == 0) {
-                // fold this partial level's counters into the control state: the
-                // barrier that follows resets them before the grid continues
-                __threadfence();
-                const Snap sn = take_snapshot(S);
-                sm.ctrl.level_min = min(sm.ctrl.level_min, sn.min);
-                sm.ctrl.alive_carry = (int64_t)sn.alive_out;
-                sm.ctrl.cont = 1;
-                sm.ctrl.solo = 0;
-                sm.ctrl.scan_target += gridDim.x;
-            }
-            __syncthreads();
-            break;
-        }
+        run_phase(A, c, sm, 0, 1);  // ends with __syncthreads (block_min_atomic)
         if (threadIdx.x == 0) {
             __threadfence();
             const Snap sn = take_snapshot(S);
-            trace_rec(S, sm.ctrl, sn, 0, (int64_t)ld_relaxed_u64(&S->arcs_walked));
-            advance(sm.ctrl, sn, p, (int)gridDim.x);
+            trace_rec(S, sm.ctrl, sn, 0);
+            advance(sm.ctrl, sn, p);
         }
         __syncthreads();
         if (sm.ctrl.phase == PH_DONE || !sm.ctrl.solo) break;
@@ -1034,6 +922,7 @@ __device__ __forceinline__ void init_ctrl(Ctrl &z)
     z.level_min = INT_MAX;
     z.alive_sel = -1;
     z.src_sel = -1;
+    z.light = 0;
 }
 
 __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
@@ -1045,7 +934,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
     if (threadIdx.x == 0) init_ctrl(sm.ctrl);
     phase_init(A, sm);
     grid_barrier(A, sm);
-    if (threadIdx.x == 0) advance(sm.ctrl, sm.snap, p, (int)gridDim.x);
+    if (threadIdx.x == 0) advance(sm.ctrl, sm.snap, p);
     __syncthreads();
     while (true) {
         if (sm.ctrl.phase == PH_DONE) break;
@@ -1063,12 +952,12 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
             }
         } else {
             const Ctrl c = sm.ctrl;
-            phase_level(A, c, sm, blockIdx.x, gridDim.x);
+            run_phase(A, c, sm, blockIdx.x, gridDim.x);
             grid_barrier(A, sm);
             if (threadIdx.x == 0) {
-                if (blockIdx.x == 0) trace_rec(S, sm.ctrl, sm.snap, 1, (int64_t)ld_relaxed_u64(&S->arcs_walked));
+                if (blockIdx.x == 0) trace_rec(S, sm.ctrl, sm.snap, 1);
                 sm.ctrl.st_bar++;
-                advance(sm.ctrl, sm.snap, p, (int)gridDim.x);
+                advance(sm.ctrl, sm.snap, p);
             }
         }
         __syncthreads();
@@ -1077,9 +966,8 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
 }
 
 // -------------------------------------------- host-driven ablation kernels
-// (KCORE_ALGO_HOSTLOOP: the paper's Alg. 1 structure -- one launch per level
-// and a host read-back of the phase after each.  No solo levels.
-// Launched cooperatively: the pool loop waits on other CTAs of the launch.)
+// (KCORE_ALGO_HOSTLOOP: the paper's Alg. 1 structure -- one launch per phase
+// and a host read-back of the phase after each.  No solo phases.)
 __global__ void __launch_bounds__(kBlock, 1) k_phase(KArgs A)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
@@ -1092,18 +980,18 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(KArgs A)
     __syncthreads();
     const Ctrl c = sm.ctrl;
     if (c.phase == PH_INIT) phase_init(A, sm);
-    else if (c.phase == PH_LEVEL) phase_level(A, c, sm, blockIdx.x, gridDim.x);
+    else run_phase(A, c, sm, blockIdx.x, gridDim.x);
 }
 
-__global__ void k_leader(KArgs A, int32_t *phase_out, int32_t nblk)
+__global__ void k_leader(KArgs A, int32_t *phase_out)
 {
     State *S = A.S;
     const Params p = S->prm;
     Ctrl c = S->pub;
     const Snap sn = take_snapshot(S);
-    trace_rec(S, c, sn, 1, (int64_t)S->arcs_walked);
+    trace_rec(S, c, sn, 1);
     c.st_bar++;
-    advance(c, sn, p, nblk);
+    advance(c, sn, p);
     S->pub = c;
     *phase_out = c.phase;
 }
@@ -1112,13 +1000,10 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
                              int64_t *trace, int64_t *trace_cta, int64_t trace_cap)
 {
     if (threadIdx.x == 0 && blockIdx.x == 0) {
+        S->gq_tail = 0ULL;
         S->ord_tail = 0ULL;
         S->alive_out = 0ULL;
         S->min_next = INT_MAX;
-        S->pool_tail = 0ULL;
-        S->pool_claim = 0ULL;
-        S->pool_done = 0ULL;
-        S->scans_done = 0ULL;
         S->bar_count = 0u;
         S->bar_gen = 0u;
         S->arcs_walked = 0ULL;

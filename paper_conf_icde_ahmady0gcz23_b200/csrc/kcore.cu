@@ -62,16 +62,15 @@ struct Carve {
     State *S;
     int32_t *order;
     uint32_t *claimed;
-    int32_t *pool_v, *pool_len;
-    int64_t *pool_beg, *pool_P;
-    int64_t pool_cap;
+    int32_t *gq_v;
+    int64_t *gq_beg, *gq_arc;
     int32_t *alive0, *alive1;
     int32_t *seg0, *seg1;
 };
 
 constexpr int kMaxSeg = 16384;  // one alive-list segment per warp of the persistent grid
 
-size_t carve(void *base, int64_t n, int64_t m, Carve *c)
+size_t carve(void *base, int64_t n, Carve *c)
 {
     size_t off = 0;
     auto take = [&](size_t bytes) {
@@ -84,14 +83,9 @@ size_t carve(void *base, int64_t n, int64_t m, Carve *c)
     t.S = (State *)take(sizeof(State));
     t.order = (int32_t *)take(sizeof(int32_t) * nn);
     t.claimed = (uint32_t *)take(sizeof(uint32_t) * ((nn + 31) / 32));
-    // a vertex enters the pool at most once per level phase it is processed in;
-    // with the local-round cap a frontier may be pushed back once: 2n bounds it
-    (void)m;
-    t.pool_cap = 2 * (int64_t)nn + 1024;
-    t.pool_v = (int32_t *)take(sizeof(int32_t) * (size_t)t.pool_cap);
-    t.pool_len = (int32_t *)take(sizeof(int32_t) * (size_t)t.pool_cap);
-    t.pool_beg = (int64_t *)take(sizeof(int64_t) * (size_t)t.pool_cap);
-    t.pool_P = (int64_t *)take(sizeof(int64_t) * (size_t)t.pool_cap);
+    t.gq_v = (int32_t *)take(sizeof(int32_t) * nn);
+    t.gq_beg = (int64_t *)take(sizeof(int64_t) * nn);
+    t.gq_arc = (int64_t *)take(sizeof(int64_t) * (nn + 1));
     t.alive0 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
@@ -129,7 +123,7 @@ extern "C" size_t kcore_workspace_size(int64_t n, int64_t m)
 {
     (void)m;
     if (n < 0) return 0;
-    return carve(nullptr, n, m, nullptr);
+    return carve(nullptr, n, nullptr);
 }
 
 extern "C" const char *kcore_strerror(int status)
@@ -179,7 +173,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     const int bloom = (opt && (opt->flags & KCORE_FLAG_NO_BLOOM)) ? 0 : 1;
     const size_t smem = sizeof(Smem);
 
-    const size_t need = carve(nullptr, n, m, nullptr);
+    const size_t need = carve(nullptr, n, nullptr);
     void *ws = nullptr;
     bool own_ws = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
@@ -194,17 +188,15 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaMallocAsync(&ws, need, st));
         own_ws = true;
     }
-    carve(ws, n, m, &cv);
+    carve(ws, n, &cv);
     A.rowptr = rowptr;
     A.colidx = colidx;
     A.deg = core_out;
     A.order = (opt && opt->order_out) ? cv.order : nullptr;  // record the peel order only on request
     A.claimed = cv.claimed;
-    A.pool_v = cv.pool_v;
-    A.pool_beg = cv.pool_beg;
-    A.pool_len = cv.pool_len;
-    A.pool_P = cv.pool_P;
-    A.pool_cap = cv.pool_cap;
+    A.gq_v = cv.gq_v;
+    A.gq_beg = cv.gq_beg;
+    A.gq_arc = cv.gq_arc;
     A.alive[0] = cv.alive0;
     A.alive[1] = cv.alive1;
     A.seg_len[0] = cv.seg0;
@@ -232,9 +224,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         int32_t ph = PH_INIT;
         int guard = 0;
         while (ph != PH_DONE) {
-            void *pargs[] = {&A};
-            KC_CUDA(cudaLaunchCooperativeKernel((const void *)k_phase, dim3(grid), dim3(kBlock), pargs, smem, st));
-            k_leader<<<1, 1, 0, st>>>(A, d_phase, grid);
+            k_phase<<<grid, kBlock, smem, st>>>(A);
+            k_leader<<<1, 1, 0, st>>>(A, d_phase);
             KC_CUDA(cudaGetLastError());
             KC_CUDA(cudaMemcpyAsync(&ph, d_phase, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
             KC_CUDA(cudaStreamSynchronize(st));
@@ -258,7 +249,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         stats->scanned = c.st_scanned;
         stats->arcs_walked = (int64_t)hS.arcs_walked;
         stats->compactions = c.st_compact;
-        stats->hub_arcs = c.st_pool;
+        stats->hub_arcs = c.st_hubarcs;
         stats->kmax = c.st_kmax;
         stats->grid_blocks = algo == KCORE_ALGO_PERSISTENT ? grid : grid;
         stats->block_threads = kBlock;
