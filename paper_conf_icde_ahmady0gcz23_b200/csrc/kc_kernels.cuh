@@ -321,7 +321,7 @@ __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gc
 // valid peel order -- the I4 certificate), then send each to the local next
 // frontier `nx` if it is small and fits the sub-round's arc budget, else to
 // the global queue.  Zero-degree vertices are only recorded.
-__device__ __forceinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool won, int32_t v,
+__device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool won, int32_t v,
                                           int32_t dv, int64_t bv, int nx, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
@@ -455,12 +455,11 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
         else if (lane == 31) nxt = LOCAL ? sm.lpre[j + 1] : ld_cg_i64(A.gq_arc + j + 1);
         const int64_t limit = min(a1, __shfl_sync(kFull, nxt, 31));
         const int64_t bmq = wbeg - wq;  // colidx index of arc x in this entry = bmq + x
-        while (a < limit) {
-            // window starts relative to this batch, clamped to int32
-            const int64_t rq = wq - a;
+        // colidx targets of the batch at arc ab (window search relative to ab)
+        auto gather = [&](int64_t ab, int32_t *out) {
+            const int64_t rq = wq - ab;
             const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
-            const int32_t lim = (int32_t)min((int64_t)kBatch, limit - a);
-            int32_t u[kUnroll];
+            const int32_t lim = (int32_t)min((int64_t)kBatch, limit - ab);
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
                 const int32_t my = r * 32 + lane;
@@ -471,8 +470,19 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
                     if (q <= my) pos += bs;
                 }
                 const int64_t off = __shfl_sync(kFull, bmq, pos);
-                u[r] = (my < lim) ? ld_stream_i32(A.colidx + off + a + my) : -1;
+                out[r] = (my < lim) ? ld_stream_i32(A.colidx + off + ab + my) : -1;
             }
+        };
+        // software pipeline: the next batch's colidx loads (HBM) are in flight
+        // while this batch's deg loads and atomics (L2) complete
+        int32_t un[kUnroll];
+        if (a < limit) gather(a, un);
+        while (a < limit) {
+            int32_t u[kUnroll];
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) u[r] = un[r];
+            const int64_t an = a + kBatch;
+            if (an < limit) gather(an, un);
             if (use_bloom) {
 #pragma unroll
                 for (int r = 0; r < kUnroll; r++)
@@ -492,7 +502,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
                 else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
             }
             if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, gcnt);
-            a += kBatch;
+            a = an;
         }
         a = limit;
         i += 32;

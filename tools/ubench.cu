@@ -5,6 +5,7 @@
 #include <cstdint>
 #include <vector>
 #include <algorithm>
+#include <string>
 #include <cuda_runtime.h>
 
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { printf("CUDA %s at %d\n", cudaGetErrorString(e), __LINE__); exit(1);} } while (0)
@@ -136,8 +137,44 @@ __global__ void k_clock_rate(uint64_t *t, long long *c, int spin)
     t[0] = t1 - t0; c[0] = c1 - c0;
 }
 
-int main()
+__global__ void k_contend(unsigned long long *ctr, int iters, int spread, unsigned long long *sink)
 {
+    // one lane per warp does `iters` returning atomics on one of `spread` addresses (128 B apart)
+    if ((threadIdx.x & 31) != 0) return;
+    const int w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    unsigned long long acc = 0;
+    unsigned long long *p = ctr + (size_t)(w % spread) * 16;
+    for (int i = 0; i < iters; i++) acc += atomicAdd(p, 64ULL);
+    if (acc == 12345) sink[0] = acc;
+}
+
+int contention()
+{
+    int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
+    unsigned long long *ctr, *sink;
+    CK(cudaMalloc(&ctr, 16 * 8 * 4096)); CK(cudaMalloc(&sink, 64));
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    for (int spread : {1, 8, 148, 4096}) {
+        for (int wpb : {1, 24}) {
+            CK(cudaMemset(ctr, 0, 16 * 8 * 4096));
+            const int iters = 200;
+            for (int rep = 0; rep < 2; rep++) {
+                cudaEventRecord(e0);
+                k_contend<<<sms, 32 * wpb>>>(ctr, iters, spread, sink);
+                cudaEventRecord(e1); CK(cudaEventSynchronize(e1));
+            }
+            float ms; cudaEventElapsedTime(&ms, e0, e1);
+            const double ops = (double)sms * wpb * iters;
+            printf("returning atomicAdd, %4d addresses, %5d warps: %.1f Mops/s, %.0f ns per op per warp\n", spread,
+                   sms * wpb, ops / ms / 1e3, ms * 1e6 / iters);
+        }
+    }
+    return 0;
+}
+
+int main(int argc, char **argv)
+{
+    if (argc > 1 && std::string(argv[1]) == "contention") return contention();
     int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
     int l2; CK(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, 0));
     printf("SMs=%d L2=%d MB\n", sms, l2 >> 20);
