@@ -22,7 +22,7 @@ import os
 from dataclasses import dataclass
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "lib", "libkcore.so")
+LIB_PATH = os.environ.get("KCORE_LIB") or os.path.join(_HERE, "lib", "libkcore.so")  # override: tuning sweeps
 
 KCORE_OK = 0
 KCORE_EINVAL = -1

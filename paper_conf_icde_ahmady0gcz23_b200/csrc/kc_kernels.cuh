@@ -45,19 +45,40 @@
 
 namespace kc {
 
-constexpr int kBlock = 768;
+#ifndef KC_BLOCK
+#define KC_BLOCK 768
+#endif
+constexpr int kBlock = KC_BLOCK;
 constexpr int kWarps = kBlock / 32;
-constexpr int kScanItems = 8;        // alive-list entries per lane per warp step
+#ifndef KC_SCAN_ITEMS
+#define KC_SCAN_ITEMS 8
+#endif
+constexpr int kScanItems = KC_SCAN_ITEMS;        // alive-list entries per lane per warp step
 constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)
 // CTA-local routing budgets (arcs), chosen per level from the size of the
 // previous level: light levels keep their BFS local, heavy ones go grid-wide.
 constexpr int kLightLevelArcs = 4 << 20;
 constexpr int kHubLight = 32768, kSubLight = 32768, kPhaseLight = 262144;
-constexpr int kHubHeavy = 8192, kSubHeavy = 8192, kPhaseHeavy = 16384;
-constexpr int kGStage = 64;          // per-warp global-queue stage (any size; flushed 32 at a time)
+#ifndef KC_HUB
+#define KC_HUB 8192
+#endif
+#ifndef KC_SUB
+#define KC_SUB 8192
+#endif
+#ifndef KC_PHASE
+#define KC_PHASE 16384
+#endif
+constexpr int kHubHeavy = KC_HUB, kSubHeavy = KC_SUB, kPhaseHeavy = KC_PHASE;
+#ifndef KC_GSTAGE
+#define KC_GSTAGE 64
+#endif
+constexpr int kGStage = KC_GSTAGE;          // per-warp global-queue stage (any size; flushed 32 at a time)
 constexpr int kBloomBits = 1 << 20;  // 128 KB
 constexpr int kBloomWords = kBloomBits / 32;
-constexpr int kBloomMaxA = 1 << 18;  // build only for alive lists up to this length
+#ifndef KC_BLOOM_MAXA
+#define KC_BLOOM_MAXA (1 << 18)
+#endif
+constexpr int kBloomMaxA = KC_BLOOM_MAXA;  // build only for alive lists up to this length
 constexpr int kUnroll = 4;  // arcs per lane in flight per batch (handle_hits assumes 4)
 constexpr int kBatch = 32 * kUnroll;
 constexpr int kTraceFields = 8;

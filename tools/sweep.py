@@ -1,0 +1,24 @@
+"""Time every library variant in paper_conf_icde_ahmady0gcz23_b200/lib/variants on C1..C4
+(one subprocess per variant; development aid)."""
+import glob, json, os, subprocess, sys
+VAR = sorted(glob.glob('paper_conf_icde_ahmady0gcz23_b200/lib/variants/*.so'))
+names = sys.argv[1:] or ["C1", "C2", "C3", "C4"]
+CODE = r'''
+import sys, json, torch
+sys.path.insert(0, '.')
+import kcgen, paper_conf_icde_ahmady0gcz23_b200 as kc
+out = {}
+for name in %r:
+    r, c = kcgen.generate_device(kcgen.CONFIGS[name])
+    ws = torch.empty(kc.kcore_workspace_size(r.numel()-1, c.numel()), dtype=torch.uint8, device='cuda')
+    for _ in range(2): kc.kcore_decompose(r, c, workspace=ws, stats=True)
+    ms = sorted(kc.kcore_decompose(r, c, workspace=ws, stats=True)[1].kernel_ms for _ in range(5))
+    out[name] = round(ms[2], 3)
+    del r, c; torch.cuda.empty_cache()
+print(json.dumps(out))
+''' % (names,)
+for v in VAR:
+    env = dict(os.environ, KCORE_LIB=os.path.abspath(v))
+    p = subprocess.run([sys.executable, "-c", CODE], env=env, capture_output=True, text=True, timeout=600)
+    res = p.stdout.strip().splitlines()[-1] if p.stdout.strip() else p.stderr[-300:]
+    print(f"{os.path.basename(v):12s} {res}", flush=True)

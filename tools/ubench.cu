@@ -148,6 +148,33 @@ __global__ void k_contend(unsigned long long *ctr, int iters, int spread, unsign
     if (acc == 12345) sink[0] = acc;
 }
 
+int hotset()
+{
+    int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
+    int *d, *sink;
+    CK(cudaMalloc(&d, 64 << 20)); CK(cudaMemset(d, 0, 64 << 20)); CK(cudaMalloc(&sink, 64));
+    cudaEvent_t e0, e1; cudaEventCreate(&e0); cudaEventCreate(&e1);
+    for (int bits : {24, 20, 17, 14, 12}) {
+        const uint32_t mask = (1u << bits) - 1;
+        for (int mode = 0; mode < 3; mode++) {
+            const int grid = sms * 4, block = 256;
+            const long long per = 2048;
+            for (int rep = 0; rep < 2; rep++) {
+                cudaEventRecord(e0);
+                if (mode == 0) k_scatter<0><<<grid, block>>>(d, mask, per, sink);
+                if (mode == 1) k_scatter<1><<<grid, block>>>(d, mask, per, sink);
+                if (mode == 2) k_scatter<2><<<grid, block>>>(d, mask, per, sink);
+                cudaEventRecord(e1); CK(cudaEventSynchronize(e1));
+            }
+            float ms; cudaEventElapsedTime(&ms, e0, e1);
+            const double ops = (double)grid * block * per;
+            printf("%s over %8u addresses: %.1f Gops/s\n", mode == 0 ? "ld.cg      " : (mode == 1 ? "atomic ret " : "atomic nort"),
+                   mask + 1, ops / ms / 1e6);
+        }
+    }
+    return 0;
+}
+
 int contention()
 {
     int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
@@ -175,6 +202,7 @@ int contention()
 int main(int argc, char **argv)
 {
     if (argc > 1 && std::string(argv[1]) == "contention") return contention();
+    if (argc > 1 && std::string(argv[1]) == "hotset") return hotset();
     int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
     int l2; CK(cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, 0));
     printf("SMs=%d L2=%d MB\n", sms, l2 >> 20);
