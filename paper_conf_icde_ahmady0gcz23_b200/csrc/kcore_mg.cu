@@ -132,20 +132,35 @@ __device__ __forceinline__ bool decrement(RankView &R, int64_t i, int k, int &lm
     return false;
 }
 
+// Frontier vertices with more than kBig arcs are walked by a whole CTA
+// (BIG=true launch), the rest by one warp each (BIG=false launch).
+constexpr int64_t kBig = 4096;
+
+template <bool BIG>
+__device__ __forceinline__ bool mg_unit(const RankView &R, int64_t f, int64_t &a0, int64_t &a1)
+{
+    const int32_t v = R.F[f];
+    a0 = R.rp[v] - R.rp0;
+    a1 = R.rp[v + 1] - R.rp0;
+    return BIG ? (a1 - a0 > kBig) : (a1 - a0 <= kBig);
+}
+
 // pass 1: remote decrements per destination (shared-memory histogram)
+template <bool BIG>
 __global__ void k_mg_count(RankView R, Owners O, int64_t fcnt, int32_t self)
 {
     __shared__ unsigned long long hist[kMaxRanks];
     for (int d = threadIdx.x; d < O.nranks; d += blockDim.x) hist[d] = 0;
     __syncthreads();
-    const int lane = threadIdx.x & 31;
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int64_t unit = BIG ? blockIdx.x : (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    const int64_t units = BIG ? gridDim.x : (((int64_t)gridDim.x * blockDim.x) >> 5);
+    const int64_t first = BIG ? wib * 32 : 0, step = BIG ? blockDim.x : 32;
     const int64_t lo_own = O.start[self], hi_own = O.start[self + 1];
-    for (int64_t f = warp; f < fcnt; f += nw) {
-        const int32_t v = R.F[f];
-        const int64_t a0 = R.rp[v] - R.rp0, a1 = R.rp[v + 1] - R.rp0;
-        for (int64_t a = a0 + lane; a < a1; a += 32) {
+    for (int64_t f = unit; f < fcnt; f += units) {
+        int64_t a0, a1;
+        if (!mg_unit<BIG>(R, f, a0, a1)) continue;
+        for (int64_t a = a0 + first + lane; a < a1; a += step) {
             const int64_t u = R.ci[a];
             if (u < lo_own || u >= hi_own) atomicAdd(&hist[owner_of(O, u)], 1ULL);
         }
@@ -158,17 +173,19 @@ __global__ void k_mg_count(RankView R, Owners O, int64_t fcnt, int32_t self)
 // pass 2: apply owned decrements, pack remote ones at off[d] + cursor
 struct Offs { unsigned long long off[kMaxRanks]; };
 
+template <bool BIG>
 __global__ void k_mg_fill(RankView R, Owners O, Offs S, int64_t fcnt, int32_t self, int k)
 {
-    const int lane = threadIdx.x & 31;
-    const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int64_t unit = BIG ? blockIdx.x : (((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5);
+    const int64_t units = BIG ? gridDim.x : (((int64_t)gridDim.x * blockDim.x) >> 5);
+    const int64_t first = BIG ? wib * 32 : 0, step = BIG ? blockDim.x : 32;
     const int64_t lo_own = O.start[self], hi_own = O.start[self + 1];
     int lmin = INT_MAX;
-    for (int64_t f = warp; f < fcnt; f += nw) {
-        const int32_t v = R.F[f];
-        const int64_t a0 = R.rp[v] - R.rp0, a1 = R.rp[v + 1] - R.rp0;
-        for (int64_t ab = a0; ab < a1; ab += 32) {
+    for (int64_t f = unit; f < fcnt; f += units) {
+        int64_t a0, a1;
+        if (!mg_unit<BIG>(R, f, a0, a1)) continue;
+        for (int64_t ab = a0 + first; ab < a1; ab += step) {
             const int64_t a = ab + lane;
             int64_t u = -1;
             if (a < a1) u = R.ci[a];
@@ -398,7 +415,10 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
             // pass 1: counts
             for (int r = 0; r < L; r++) {
                 k_mg_reset<<<1, 64, 0, st>>>(R[r].ctl, P);
-                if (fcnt[r]) k_mg_count<<<grid_for(fcnt[r] * 32), kMgBlock, 0, st>>>(R[r], O, fcnt[r], self0 + r);
+                if (fcnt[r]) {
+                    k_mg_count<false><<<grid_for(fcnt[r] * 32), kMgBlock, 0, st>>>(R[r], O, fcnt[r], self0 + r);
+                    k_mg_count<true><<<grid_for(fcnt[r] * kMgBlock), kMgBlock, 0, st>>>(R[r], O, fcnt[r], self0 + r);
+                }
                 MG_CK(cudaGetLastError());
                 MG_CK(cudaMemcpyAsync(&hc[r], R[r].ctl, sizeof(MgCtl), cudaMemcpyDeviceToHost, st));
             }
@@ -426,7 +446,10 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
             for (int r = 0; r < L; r++) {
                 Offs S;
                 for (int d = 0; d < P; d++) S.off[d] = soff[r][d];
-                if (fcnt[r]) k_mg_fill<<<grid_for(fcnt[r] * 32), kMgBlock, 0, st>>>(R[r], O, S, fcnt[r], self0 + r, k);
+                if (fcnt[r]) {
+                    k_mg_fill<false><<<grid_for(fcnt[r] * 32), kMgBlock, 0, st>>>(R[r], O, S, fcnt[r], self0 + r, k);
+                    k_mg_fill<true><<<grid_for(fcnt[r] * kMgBlock), kMgBlock, 0, st>>>(R[r], O, S, fcnt[r], self0 + r, k);
+                }
                 MG_CK(cudaGetLastError());
             }
             MG_RC(T.exchange_payload(R, send, soff, recv, roff));
