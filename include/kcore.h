@@ -73,10 +73,11 @@ typedef enum {
 typedef struct {
     int32_t algo;            /* KCORE_ALGO_*                                           */
     int32_t blocks_per_sm;   /* 0 = auto (occupancy); persistent grid = SMs x this     */
-    int32_t solo_arcs;       /* 0 = default; peel sub-rounds with <= this many arcs run */
-                             /* on ONE CTA with CTA-local sync (no grid barrier); -1 off */
-    int32_t solo_scan;       /* 0 = default; level scans over <= this many alive       */
-                             /* entries run on one CTA; -1 off                          */
+    int32_t solo_arcs;       /* > 0: HUB phases with <= this many arcs run on ONE CTA   */
+                             /* with CTA-local sync (no grid barrier); 0/-1 = off      */
+                             /* (default: off, slower on B200 -- DESIGN.md)            */
+    int32_t solo_scan;       /* > 0: levels over <= this many alive entries run on one */
+                             /* CTA; 0/-1 = off (default off)                           */
     int32_t *order_out;      /* optional DEVICE int32[n]: peel order (concatenated      */
                              /* frontiers; a degeneracy order)          */
     void *workspace;         /* optional DEVICE scratch of >= kcore_workspace_size()    */

@@ -51,7 +51,7 @@ namespace kc {
 constexpr int kBlock = KC_BLOCK;
 constexpr int kWarps = kBlock / 32;
 #ifndef KC_SCAN_ITEMS
-#define KC_SCAN_ITEMS 8
+#define KC_SCAN_ITEMS 4
 #endif
 constexpr int kScanItems = KC_SCAN_ITEMS;        // alive-list entries per lane per warp step
 constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)

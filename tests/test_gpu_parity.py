@@ -39,7 +39,7 @@ def _check(rp, ci, ref=None, **kw):
     return got
 
 
-VARIANTS = [dict(), dict(solo_arcs=-1, solo_scan=-1), dict(bloom=False), dict(algo=kc.ALGO_HOSTLOOP),
+VARIANTS = [dict(), dict(solo_arcs=16384, solo_scan=32768), dict(bloom=False), dict(algo=kc.ALGO_HOSTLOOP),
             dict(solo_arcs=1 << 30, solo_scan=1 << 30)]
 
 
@@ -101,7 +101,7 @@ def test_long_path_many_subrounds():
     """P_n peels from both ends: n/2 dependent sub-rounds in one level."""
     n = 100_000
     rp, ci = kcgen.csr_from_edges(n, [(i, i + 1) for i in range(n - 1)])
-    for kw in (dict(), dict(solo_arcs=-1)):
+    for kw in (dict(), dict(solo_arcs=16384, solo_scan=32768)):
         _check(rp, ci, np.ones(n, np.int32), **kw)
 
 
@@ -150,7 +150,7 @@ def test_exhaustive_union_n6():
 def test_exhaustive_union_n7():
     rp, ci = _all_graphs_union(7)
     _check(rp, ci)
-    _check(rp, ci, solo_arcs=-1)
+    _check(rp, ci, solo_arcs=16384, solo_scan=32768)
 
 
 def test_random_graphs_and_launch_shapes():
