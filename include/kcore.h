@@ -64,6 +64,9 @@ typedef enum {
 
 /* kcore_options.flags */
 #define KCORE_FLAG_NO_BLOOM 1   /* disable the shared-memory alive-set filter (ablation) */
+#define KCORE_FLAG_POOL 2       /* in-phase work pool: vertices too big for one CTA are   */
+                                /* split into items any idle warp takes in the same phase */
+                                /* (experimental; default off -- DESIGN.md)               */
 
 /* Algorithms selectable through kcore_options.algo. */
 #define KCORE_ALGO_PERSISTENT 0 /* default: one persistent kernel, device-resident loop */
@@ -89,9 +92,11 @@ typedef struct {
                              /* reported in kcore_stats.trace_len)                      */
     int32_t flags;           /* KCORE_FLAG_* bits                                        */
     int32_t reserved1;
-    int64_t *trace_cta_out;  /* optional DEVICE int64[trace_cap][grid][4]: per phase and */
+    int64_t *trace_cta_out;  /* optional DEVICE int64[trace_cap][grid][8]: per phase and */
                              /* CTA, globaltimer at {phase start, end of scan or queue  */
-                             /* walk, end of local drain, barrier arrival}              */
+                             /* walk, end of local drain, barrier arrival, local sub-  */
+                             /* rounds, arcs walked, vertices removed, largest sub-     */
+                             /* round in arcs}                                          */
     int64_t reserved[1];
 } kcore_options;
 

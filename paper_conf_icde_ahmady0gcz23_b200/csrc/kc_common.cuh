@@ -49,12 +49,29 @@ __device__ __forceinline__ int32_t ld_relaxed_i32(const int32_t *p)
 }
 
 // streaming read-only loads of the CSR (never written during a call)
+#ifdef KC_COLIDX_EVICT_FIRST
+// L2 evict-first: the adjacency stream must not push deg / code out of L2
+__device__ __forceinline__ uint64_t l2_evict_first_policy()
+{
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p)
+{
+    int32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.s32 %0, [%1], %2;"
+                 : "=r"(v) : "l"(p), "l"(l2_evict_first_policy()));
+    return v;
+}
+#else
 __device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p)
 {
     int32_t v;
     asm volatile("ld.global.nc.L1::no_allocate.s32 %0, [%1];" : "=r"(v) : "l"(p));
     return v;
 }
+#endif
 
 __device__ __forceinline__ int64_t ld_ro_i64(const int64_t *p) { return __ldg(p); }
 

@@ -82,6 +82,20 @@ constexpr int kBloomMaxA = KC_BLOOM_MAXA;  // build only for alive lists up to t
 constexpr int kUnroll = 4;  // arcs per lane in flight per batch (handle_hits assumes 4)
 constexpr int kBatch = 32 * kUnroll;
 constexpr int kTraceFields = 8;
+// Work pool: vertices too big for one CTA are split into items of about
+// kItemArcs arcs that any idle warp of the grid takes within the same phase.
+#ifndef KC_POOL_CAP
+#define KC_POOL_CAP (1 << 16)
+#endif
+constexpr int kPoolCap = KC_POOL_CAP;  // items per phase (beyond: global queue)
+#ifndef KC_ITEM
+#define KC_ITEM 256
+#endif
+constexpr int kItemArcs = KC_ITEM;
+constexpr int kItemMax = 64;          // items per vertex at most
+constexpr int kItemLenBits = 26;      // item word: ((beg + 1) << 26) | len
+constexpr unsigned long long kItemNull = 1ULL;  // a reserved slot left unused
+static_assert(kItemArcs >= kItemMax, "every item of a split vertex must be non-empty");
 
 enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
@@ -118,7 +132,7 @@ struct Params {
     int32_t solo_arcs;  // HUB phases with <= this many arcs run solo
     int32_t solo_scan;  // LEVEL phases over <= this many entries run solo
     int32_t bloom;      // 0 disables the Bloom filter
-    int32_t pad;
+    int32_t pool;       // 0 disables the work pool
 };
 
 struct State {
@@ -130,10 +144,12 @@ struct State {
     alignas(128) uint32_t bar_gen;              // grid barrier generation
     Snap snap[2];                               // counters at barrier gen, by gen & 1
     alignas(128) unsigned long long arcs_walked;
+    alignas(128) unsigned long long pool_pk;    // packed (items reserved << 32) | pending units
+    alignas(128) unsigned long long pool_head;  // next ticket
     alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
     alignas(128) Params prm;
     int64_t *trace;                             // optional [trace_cap][kTraceFields]
-    int64_t *trace_cta;                         // optional [trace_cap][grid][4]
+    int64_t *trace_cta;                         // optional [trace_cap][grid][8]
     int64_t trace_cap;
     unsigned long long trace_n;
 };
@@ -151,7 +167,8 @@ struct KArgs {
     int32_t *seg_len[2];  // entries of segment b in alive[x]: seg_len[x][b]
     int64_t seg_R;        // segment region size: segment b lives at [b*R, b*R + len)
     int32_t nseg;         // = persistent grid size
-    int32_t pad;
+    int32_t pool_on;      // 1: grid phases use the work pool (persistent kernel only)
+    unsigned long long *pool;  // [kPoolCap] item words, 0 = empty
     State *S;
     int64_t n;
 };
@@ -178,7 +195,10 @@ struct Smem {
     int32_t red_min[kWarps];
     int64_t bloom_level;
     int32_t bloom_on;
-    int32_t pad;
+    int32_t pool_on;             // this phase uses the work pool (grid-uniform)
+    int32_t pool_done;           // pool drained (set by any warp of this CTA)
+    int32_t pad3;
+    unsigned long long pool_arcs;  // arcs walked from pool items by this CTA this phase
     Ctrl ctrl;
     Snap snap;
     uint32_t bloom[kBloomWords];
@@ -206,6 +226,32 @@ __device__ __forceinline__ unsigned long long globaltimer()
     return t;
 }
 
+#ifdef KC_PROBE
+// Development probe (variant builds only): {cta, tag, globaltimer, value}.
+__device__ unsigned long long g_probe_n;
+__device__ int64_t g_probe[(1 << 22) * 4];
+#ifndef KC_PROBE_KMIN
+#define KC_PROBE_KMIN 0
+#endif
+__shared__ int s_probe_k;
+__shared__ unsigned s_probe_n;
+constexpr int kProbePerCta = (1 << 22) / 160;
+__device__ __forceinline__ void probe(int tag, int64_t val)
+{
+    if (*(volatile int *)&s_probe_k < KC_PROBE_KMIN) return;
+    const int64_t t = (int64_t)globaltimer();
+    const unsigned i = atomicAdd(&s_probe_n, 1u);
+    if (i >= (unsigned)kProbePerCta) return;
+    int64_t *r = g_probe + ((int64_t)blockIdx.x * kProbePerCta + i) * 4;
+    r[0] = blockIdx.x; r[1] = tag; r[2] = t; r[3] = val;
+}
+#define PROBE(tag, val) probe(tag, val)
+#define PROBE_W(tag, val) ((void)0)
+#else
+#define PROBE_W(tag, val) ((void)0)
+#define PROBE(tag, val) ((void)0)
+#endif
+
 __device__ __forceinline__ uint32_t bloom_h1(uint32_t v) { return (v * 0x9E3779B1u) >> 12; }
 __device__ __forceinline__ uint32_t bloom_h2(uint32_t v) { return ((v ^ (v >> 15)) * 0x85EBCA6Bu) >> 12; }
 
@@ -223,7 +269,17 @@ __device__ __forceinline__ void cta_time(const KArgs &A, const Ctrl &c, int slot
     if (threadIdx.x != 0 || c.solo) return;
     State *S = A.S;
     if (!S->trace_cta || c.st_bar >= S->trace_cap) return;
-    S->trace_cta[(c.st_bar * gridDim.x + blockIdx.x) * 4 + slot] = (int64_t)globaltimer();
+    S->trace_cta[(c.st_bar * gridDim.x + blockIdx.x) * 8 + slot] = (int64_t)globaltimer();
+}
+
+// Per-CTA counters of the current phase (trace mode only): slot 4 local
+// sub-rounds, 5 arcs walked, 6 vertices removed, 7 largest sub-round (arcs).
+__device__ __forceinline__ void cta_count(const KArgs &A, const Ctrl &c, int slot, int64_t val)
+{
+    if (threadIdx.x != 0 || c.solo) return;
+    State *S = A.S;
+    if (!S->trace_cta || c.st_bar >= S->trace_cap) return;
+    S->trace_cta[(c.st_bar * gridDim.x + blockIdx.x) * 8 + slot] = val;
 }
 
 // CTA-wide min, then one atomicMin per CTA
@@ -336,6 +392,70 @@ __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gc
     gcnt = 0;
 }
 
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long *p, unsigned long long v)
+{
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+// Push the vertices of the lanes where `want` into the work pool, each split
+// into ceil(d / kItemArcs) items (at most kItemMax).  One packed atomic
+// reserves the slots and adds them to the pending count before any item is
+// visible.  Returns true for lanes whose vertex did not fit (pool full for
+// this phase): the caller sends those to the global queue.
+__device__ __noinline__ bool pool_push(const KArgs &A, bool want, int32_t dv, int64_t bv)
+{
+    const int lane = threadIdx.x & 31;
+    if (__ballot_sync(kFull, want) == 0) return false;
+    int nj = 0;
+    if (want) nj = min((dv + kItemArcs - 1) / kItemArcs, kItemMax);
+    int incl = nj;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int t = __shfl_up_sync(kFull, incl, o);
+        if (lane >= o) incl += t;
+    }
+    const int tot = __shfl_sync(kFull, incl, 31);
+    const int ex = incl - nj;
+    unsigned long long base = 0;
+    int ok = 0;
+    if (lane == 0) {
+        const unsigned long long old =
+            atomicAdd(&A.S->pool_pk, ((unsigned long long)tot << 32) | (unsigned long long)tot);
+        base = old >> 32;
+        PROBE(20, (int64_t)((base << 16) | (unsigned long long)tot));
+        if (base + (unsigned long long)tot <= (unsigned long long)kPoolCap) ok = 1;
+        else atomicAdd(&A.S->pool_pk, 0ULL - (unsigned long long)tot);  // not pending after all
+        __threadfence();
+    }
+    base = __shfl_sync(kFull, base, 0);
+    ok = __shfl_sync(kFull, ok, 0);
+    for (int x0 = 0; x0 < tot; x0 += 32) {
+        const int x = x0 + lane;
+        int pos = 0;
+#pragma unroll
+        for (int bs = 16; bs >= 1; bs >>= 1) {
+            const int q = __shfl_sync(kFull, ex, pos + bs);
+            if (q <= x) pos += bs;
+        }
+        const int njo = __shfl_sync(kFull, nj, pos);
+        const int dvo = __shfl_sync(kFull, dv, pos);
+        const int exo = __shfl_sync(kFull, ex, pos);
+        const int64_t bvo = __shfl_sync(kFull, bv, pos);
+        if (x < tot && base + (unsigned long long)x < (unsigned long long)kPoolCap) {
+            unsigned long long word = kItemNull;
+            if (ok) {
+                const int per = (dvo + njo - 1) / njo;
+                const int ib = (x - exo) * per;
+                const int il = min(per, dvo - ib);
+                word = ((unsigned long long)(bvo + ib + 1) << kItemLenBits) | (unsigned long long)il;
+            }
+            st_relaxed_u64(A.pool + base + x, word);
+        }
+    }
+    __syncwarp();
+    return want && !ok;
+}
+
 // Route claimed vertices (one per lane where `won`): reserve their slots in
 // the removal order right away (a vertex is claimed only after every vertex
 // whose processing made it reach k was claimed, so claim-time slots form a
@@ -359,7 +479,7 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
             atomicAdd(&sm.removed, __popc(b));
         }
     }
-    const bool cand = won && dv > 0 && dv <= sm.bud_hub;
+    const bool cand = won && dv > 0 && dv <= sm.bud_hub && nx >= 0;  // nx < 0: no local list
     const unsigned bc = __ballot_sync(kFull, cand);
     bool wantl = false;
     int lbase = 0;
@@ -392,6 +512,7 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
             tog = true;
         }
     }
+    if (sm.pool_on) tog = pool_push(A, tog, dv, bv);
     const unsigned bg = __ballot_sync(kFull, tog);
     if (bg) {
         const int c = __popc(bg);
@@ -464,6 +585,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
     }
     int64_t i = lo;
     int64_t a = a0;
+    if (LOCAL && threadIdx.x == 0) PROBE_W(10, a1 - a0);
     while (a < a1) {
         const int64_t j = i + lane;
         int64_t wq = LLONG_MAX, wbeg = 0;
@@ -522,7 +644,9 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
                 else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
                 else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
             }
+            if (LOCAL && threadIdx.x == 0) PROBE_W(12, a);
             if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, gcnt);
+            if (LOCAL && threadIdx.x == 0) PROBE_W(13, __popc(hm));
             a = an;
         }
         a = limit;
@@ -533,13 +657,14 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
 // Drain this CTA's local frontier (list `cur`) breadth-first with CTA-local
 // sub-rounds.  Returns the number of arcs walked.
 __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, bool use_bloom,
-                               int &lmin, int &gcnt)
+                               int &lmin, int &gcnt, int64_t *subs = nullptr, int64_t *tmax = nullptr)
 {
     const int wib = threadIdx.x >> 5;
     int64_t walked = 0;
     while (true) {
         __syncthreads();
         const int L = min(sm.lcnt[cur], kLCap);
+        if (threadIdx.x == 0) PROBE(1, L);
         if (L == 0) break;
         // arc prefix of the list
         const int64_t dv = threadIdx.x < L ? (int64_t)sm.ld[cur][threadIdx.x] : 0;
@@ -549,16 +674,110 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         const int nx = cur ^ 1;
         if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; sm.larc[nx] = 0; }
         __syncthreads();
+        if (threadIdx.x == 0) PROBE(2, T);
         int64_t C = (T + kWarps - 1) / kWarps;
         C = ((C + kBatch - 1) / kBatch) * kBatch;
         const int64_t a0 = (int64_t)wib * C;
         if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, lmin, gcnt);
         walked += T;
+        if (subs) { *subs += 1; *tmax = max(*tmax, T); }
+        if (threadIdx.x == 0) PROBE(3, sm.lcnt[nx]);
         __syncthreads();
         if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
         cur = nx;
     }
     return walked;
+}
+
+// One pool item: arcs [beg, beg+len) walked by one warp; hits go back to
+// the pool (or the global queue when it is full).
+__device__ __forceinline__ void walk_item(const KArgs &A, Smem &sm, const int k, int64_t beg, int len,
+                                          int &lmin, int &gcnt)
+{
+    const int lane = threadIdx.x & 31;
+    for (int a = 0; a < len; a += kBatch) {
+        int32_t u[kUnroll];
+#pragma unroll
+        for (int r = 0; r < kUnroll; r++) {
+            const int x = a + r * 32 + lane;
+            u[r] = x < len ? ld_stream_i32(A.colidx + beg + x) : -1;
+        }
+        int32_t d[kUnroll];
+#pragma unroll
+        for (int r = 0; r < kUnroll; r++) d[r] = u[r] >= 0 ? ld_cg_i32(A.deg + u[r]) : -1;
+        int old[kUnroll];
+#pragma unroll
+        for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
+        unsigned hm = 0;
+#pragma unroll
+        for (int r = 0; r < kUnroll; r++) {
+            if (old[r] == k + 1) hm |= 1u << r;
+            else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
+            else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
+        }
+        if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, -1, u[0], u[1], u[2], u[3], hm, gcnt);
+    }
+}
+
+// Take pool items until the phase's pending count (one unit per CTA until
+// its own scan + local drain is done, plus one per pushed item until it is
+// walked) reaches zero.  Each warp holds one ticket = one slot; lane 0 polls
+// the slot and, every few polls, the pending count.
+__device__ void pool_consume(const KArgs &A, Smem &sm, const int k, int &lmin, int &gcnt)
+{
+    const int lane = threadIdx.x & 31;
+    State *S = A.S;
+    volatile int32_t *done = &sm.pool_done;
+    unsigned long long walked = 0;
+    while (true) {
+        unsigned long long w = 0;
+        if (lane == 0) {
+            const unsigned long long t = atomicAdd(&S->pool_head, 1ULL);
+            unsigned spins = 0;
+            while (true) {
+                if (t < (unsigned long long)kPoolCap) {
+                    w = ld_relaxed_u64(A.pool + t);
+                    if (w) break;
+                }
+                if (*done) break;
+                if ((++spins & 3u) == 0u && (uint32_t)ld_relaxed_u64(&S->pool_pk) == 0u) {
+                    *done = 1;
+                    break;
+                }
+                __nanosleep(64);
+            }
+            if (w) { st_relaxed_u64(A.pool + t, 0ULL); PROBE(21, (int64_t)t); }
+            else if (threadIdx.x == 0) PROBE(23, (int64_t)t);
+        }
+        w = __shfl_sync(kFull, w, 0);
+        if (w == 0) break;
+        if (w == kItemNull) continue;
+        const int64_t beg = (int64_t)(w >> kItemLenBits) - 1;
+        const int len = (int)(w & ((1ULL << kItemLenBits) - 1ULL));
+        walk_item(A, sm, k, beg, len, lmin, gcnt);
+        walked += (unsigned long long)len;
+        __syncwarp();
+        if (lane == 0) { atomicAdd(&S->pool_pk, ~0ULL); PROBE(22, len); }  // after this item's pushes
+    }
+    if (lane == 0 && walked) atomicAdd(&sm.pool_arcs, walked);
+}
+
+// The CTA's own unit is released once its scan / queue walk and local drain
+// are done (its pushes are already counted); then every warp takes items.
+__device__ __forceinline__ void pool_phase_tail(const KArgs &A, const Ctrl &c, Smem &sm, int &lmin, int &gcnt)
+{
+    const int wib = threadIdx.x >> 5;
+    if (!sm.pool_on) return;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(&A.S->pool_pk, ~0ULL);
+        PROBE(31, 0);
+    }
+    pool_consume(A, sm, c.k, lmin, gcnt);
+    gq_flush(A, sm, wib, gcnt);
+    __syncthreads();
+    if (threadIdx.x == 0) PROBE(32, 0);
 }
 
 // Bloom filter of the alive list at level start (built once per level).
@@ -725,24 +944,35 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     const int wib = threadIdx.x >> 5;
     int lmin = INT_MAX, gcnt = 0;
     cta_time(A, c, 0);
+#ifdef KC_PROBE
+    if (threadIdx.x == 0) s_probe_k = c.k;
+#endif
+    if (threadIdx.x == 0) PROBE(30, c.k * 4 + c.phase);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
         sm.bud_hub = c.light ? kHubLight : kHubHeavy;
         sm.bud_sub = c.light ? kSubLight : kSubHeavy;
         sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
+        sm.pool_on = (A.pool_on && nblk > 1) ? 1 : 0;
+        sm.pool_done = 0;
+        sm.pool_arcs = 0ULL;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
     __syncthreads();
     cta_time(A, c, 1);
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
-    const int64_t walked = local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
+    int64_t subs = 0, tmax = 0;
+    const int64_t walked = local_drain(A, sm, c.k, 0, bl, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
+    pool_phase_tail(A, c, sm, lmin, gcnt);
     __syncthreads();
+    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked + (int64_t)sm.pool_arcs); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
     if (threadIdx.x == 0) {
-        if (walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+        const unsigned long long wk = (unsigned long long)walked + sm.pool_arcs;
+        if (wk) atomicAdd(&A.S->arcs_walked, wk);
         if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
     }
     block_min_atomic(sm, lmin, &A.S->min_next);
@@ -759,12 +989,19 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     C = ((C + kBatch - 1) / kBatch) * kBatch;
     int lmin = INT_MAX, gcnt = 0;
     cta_time(A, c, 0);
+#ifdef KC_PROBE
+    if (threadIdx.x == 0) s_probe_k = c.k;
+#endif
+    if (threadIdx.x == 0) PROBE(30, c.k * 4 + c.phase);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.lphase = 0; sm.removed = 0; sm.fit = 0;
         sm.bud_hub = c.light ? kHubLight : kHubHeavy;
         sm.bud_sub = c.light ? kSubLight : kSubHeavy;
         sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
+        sm.pool_on = (A.pool_on && nblk > 1) ? 1 : 0;
+        sm.pool_done = 0;
+        sm.pool_arcs = 0ULL;
     }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
@@ -775,12 +1012,16 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     int64_t walked = cta_arcs;
     __syncthreads();
     cta_time(A, c, 1);
-    walked += local_drain(A, sm, c.k, 0, bl, lmin, gcnt);
+    int64_t subs = 0, tmax = 0;
+    walked += local_drain(A, sm, c.k, 0, bl, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
+    pool_phase_tail(A, c, sm, lmin, gcnt);
     __syncthreads();
+    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked + (int64_t)sm.pool_arcs); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
     if (threadIdx.x == 0) {
-        if (walked) atomicAdd(&A.S->arcs_walked, (unsigned long long)walked);
+        const unsigned long long wk = (unsigned long long)walked + sm.pool_arcs;
+        if (wk) atomicAdd(&A.S->arcs_walked, wk);
         if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
     }
     block_min_atomic(sm, lmin, &A.S->min_next);
@@ -856,7 +1097,7 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
 }
 
 // Snapshot + reset of the counters (caller guarantees nobody else touches them).
-__device__ __forceinline__ Snap take_snapshot(State *S)
+__device__ __forceinline__ Snap take_snapshot(State *S, unsigned grid)
 {
     Snap sn;
     sn.arcs = ld_relaxed_u64(&S->arcs_walked);
@@ -867,6 +1108,8 @@ __device__ __forceinline__ Snap take_snapshot(State *S)
     sn.pad = 0;
     S->alive_out = 0ULL;
     S->min_next = INT_MAX;
+    S->pool_pk = (unsigned long long)grid;  // one pending unit per CTA
+    S->pool_head = 0ULL;
     return sn;
 }
 
@@ -894,17 +1137,20 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
     cta_time(A, sm.ctrl, 3);
     if (threadIdx.x == 0) {
         State *S = A.S;
+        PROBE(33, 0);
         const uint32_t gen = ld_acquire_u32(&S->bar_gen);
         const uint32_t t = atom_add_release_u32(&S->bar_count, 1u);
+        PROBE(35, t);
         Snap sn;
         if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
             __threadfence();
-            sn = take_snapshot(S);
+            sn = take_snapshot(S, gridDim.x);
             S->snap[(gen + 1u) & 1u] = sn;
             st_release_u32(&S->bar_gen, gen + 1u);
         } else {
             while (ld_acquire_u32(&S->bar_gen) == gen) {
             }
+            PROBE(34, 0);
             const Snap *ps = &S->snap[(gen + 1u) & 1u];
             sn.arcs = ld_relaxed_u64(&ps->arcs);
             sn.gq = ld_relaxed_u64(&ps->gq);
@@ -929,11 +1175,11 @@ __device__ void solo_run(const KArgs &A, Smem &sm, const Params &p)
 {
     State *S = A.S;
     while (true) {
-        const Ctrl c = sm.ctrl;
+        const Ctrl &c = sm.ctrl;  // shared copy: no per-thread spill
         run_phase(A, c, sm, 0, 1);  // ends with __syncthreads (block_min_atomic)
         if (threadIdx.x == 0) {
             __threadfence();
-            const Snap sn = take_snapshot(S);
+            const Snap sn = take_snapshot(S, 1u);
             trace_rec(S, sm.ctrl, sn, 0);
             advance(sm.ctrl, sn, p);
         }
@@ -963,6 +1209,10 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
     State *S = A.S;
     const Params p = S->prm;
     if (threadIdx.x == 0) init_ctrl(sm.ctrl);
+#ifdef KC_PROBE
+    if (threadIdx.x == 0) { s_probe_n = 0u; s_probe_k = 0; }
+    __syncthreads();
+#endif
     phase_init(A, sm);
     grid_barrier(A, sm);
     if (threadIdx.x == 0) advance(sm.ctrl, sm.snap, p);
@@ -982,13 +1232,16 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
                 sm.ctrl = c;
             }
         } else {
-            const Ctrl c = sm.ctrl;
+            if (threadIdx.x == 0) PROBE(38, 0);
+            const Ctrl &c = sm.ctrl;  // shared copy: no per-thread spill
             run_phase(A, c, sm, blockIdx.x, gridDim.x);
             grid_barrier(A, sm);
             if (threadIdx.x == 0) {
+                PROBE(36, 0);
                 if (blockIdx.x == 0) trace_rec(S, sm.ctrl, sm.snap, 1);
                 sm.ctrl.st_bar++;
                 advance(sm.ctrl, sm.snap, p);
+                PROBE(37, 0);
             }
         }
         __syncthreads();
@@ -1009,7 +1262,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(KArgs A)
         sm.bloom_level = -1;
     }
     __syncthreads();
-    const Ctrl c = sm.ctrl;
+    const Ctrl &c = sm.ctrl;
     if (c.phase == PH_INIT) phase_init(A, sm);
     else run_phase(A, c, sm, blockIdx.x, gridDim.x);
 }
@@ -1019,7 +1272,7 @@ __global__ void k_leader(KArgs A, int32_t *phase_out)
     State *S = A.S;
     const Params p = S->prm;
     Ctrl c = S->pub;
-    const Snap sn = take_snapshot(S);
+    const Snap sn = take_snapshot(S, gridDim.x);
     trace_rec(S, c, sn, 1);
     c.st_bar++;
     advance(c, sn, p);
@@ -1038,6 +1291,8 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
         S->bar_count = 0u;
         S->bar_gen = 0u;
         S->arcs_walked = 0ULL;
+        S->pool_pk = 0ULL;
+        S->pool_head = 0ULL;
         Ctrl z;
         init_ctrl(z);
         S->pub = z;

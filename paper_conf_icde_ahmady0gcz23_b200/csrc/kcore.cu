@@ -66,6 +66,7 @@ struct Carve {
     int64_t *gq_beg, *gq_arc;
     int32_t *alive0, *alive1;
     int32_t *seg0, *seg1;
+    unsigned long long *pool;
 };
 
 constexpr int kMaxSeg = 16384;  // one alive-list segment per warp of the persistent grid
@@ -90,6 +91,7 @@ size_t carve(void *base, int64_t n, Carve *c)
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     t.seg1 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
+    t.pool = (unsigned long long *)take(sizeof(unsigned long long) * kPoolCap);
     if (c) *c = t;
     return off;
 }
@@ -141,6 +143,20 @@ extern "C" const char *kcore_strerror(int status)
     default: return "KCORE: unknown status";
     }
 }
+
+#ifdef KC_PROBE
+extern "C" int64_t kcore_probe_read(int64_t *host, int64_t cap)
+{
+    // per-CTA regions; unused records have tag 0 (cleared after each read)
+    const size_t bytes = (size_t)(1 << 22) * 4 * sizeof(int64_t);
+    if (cap < (int64_t)(1 << 22)) return -1;
+    cudaMemcpyFromSymbol(host, kc::g_probe, bytes);
+    void *dp = nullptr;
+    cudaGetSymbolAddress(&dp, kc::g_probe);
+    cudaMemset(dp, 0, bytes);
+    return (int64_t)(1 << 22);
+}
+#endif
 
 extern "C" const char *kcore_version(void) { return "kcore-b200 0.1 (sm_100a persistent peel)"; }
 
@@ -205,7 +221,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.seg_len[1] = cv.seg1;
     A.nseg = grid;
     A.seg_R = (n + A.nseg - 1) / A.nseg;
-    A.pad = 0;
+    A.pool = cv.pool;
+    A.pool_on = (algo == KCORE_ALGO_PERSISTENT && opt && (opt->flags & KCORE_FLAG_POOL)) ? 1 : 0;
     A.S = cv.S;
     A.n = n;
 
@@ -213,6 +230,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaEventCreate(&ev0));
         KC_CUDA(cudaEventCreate(&ev1));
     }
+    KC_CUDA(cudaMemsetAsync(cv.pool, 0, sizeof(unsigned long long) * kPoolCap, st));
     k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, trace,
                                    trace ? opt->trace_cta_out : nullptr, trace_cap);
     KC_CUDA(cudaGetLastError());

@@ -11,7 +11,7 @@ for name in sys.argv[2:]:
     r, c = kcgen.generate_device(kcgen.CONFIGS[name])
     cap = 20000
     tr = torch.zeros((cap, 8), dtype=torch.int64, device='cuda')
-    tc = torch.zeros((cap, 148, 4), dtype=torch.int64, device='cuda')
+    tc = torch.zeros((cap, 148, 8), dtype=torch.int64, device='cuda')
     for _ in range(2):
         tc.zero_()
         core, st = kc.kcore_decompose(r, c, trace=tr, trace_cta=tc, stats=True)

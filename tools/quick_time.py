@@ -12,7 +12,7 @@ for name in names:
     torch.cuda.synchronize()
     tg = time.time() - t0
     n = r.numel() - 1; m = c.numel()
-    for kw in (dict(), dict(solo_arcs=-1)):
+    for kw in (dict(),):
         ws = torch.empty(kc.kcore_workspace_size(n, m), dtype=torch.uint8, device='cuda')
         for i in range(3):
             core, st = kc.kcore_decompose(r, c, workspace=ws, stats=True, **kw)

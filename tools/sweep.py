@@ -2,7 +2,8 @@
 (one subprocess per variant; development aid)."""
 import glob, json, os, subprocess, sys
 VAR = sorted(glob.glob('paper_conf_icde_ahmady0gcz23_b200/lib/variants/*.so'))
-names = sys.argv[1:] or ["C1", "C2", "C3", "C4"]
+names = [a for a in sys.argv[1:] if not a.startswith("--kw=")] or ["C1", "C2", "C3", "C4"]
+KWS = [eval(a[5:]) for a in sys.argv[1:] if a.startswith("--kw=")] or [{}]
 CODE = r'''
 import sys, json, torch
 sys.path.insert(0, '.')
@@ -11,12 +12,13 @@ out = {}
 for name in %r:
     r, c = kcgen.generate_device(kcgen.CONFIGS[name])
     ws = torch.empty(kc.kcore_workspace_size(r.numel()-1, c.numel()), dtype=torch.uint8, device='cuda')
-    for _ in range(2): kc.kcore_decompose(r, c, workspace=ws, stats=True)
-    ms = sorted(kc.kcore_decompose(r, c, workspace=ws, stats=True)[1].kernel_ms for _ in range(5))
-    out[name] = round(ms[2], 3)
+    for kw in %r:
+        for _ in range(2): kc.kcore_decompose(r, c, workspace=ws, stats=True, **kw)
+        ms = sorted(kc.kcore_decompose(r, c, workspace=ws, stats=True, **kw)[1].kernel_ms for _ in range(5))
+        out[name + (str(kw) if kw else '')] = round(ms[2], 3)
     del r, c; torch.cuda.empty_cache()
 print(json.dumps(out))
-''' % (names,)
+''' % (names, KWS)
 for v in VAR:
     env = dict(os.environ, KCORE_LIB=os.path.abspath(v))
     p = subprocess.run([sys.executable, "-c", CODE], env=env, capture_output=True, text=True, timeout=600)

@@ -11,11 +11,12 @@ names = sys.argv[1:] or ["C4"]
 for name in names:
     r, c = kcgen.generate_device(kcgen.CONFIGS[name])
     n = r.numel() - 1
-    for kw in (dict(), dict(solo_arcs=-1, solo_scan=-1), dict(bloom=False)):
+    for kw in (dict(),):
         tr = torch.zeros((400000, 8), dtype=torch.int64, device='cuda')
         for _ in range(2):
             core, st = kc.kcore_decompose(r, c, trace=tr, stats=True, **kw)
         T = tr[:st.trace_len].cpu().numpy()
+        if len(sys.argv) > 0: np.save(f'gpurun_out/trace_{name}.npy', T)
         t = T[:, 0]
         dt = np.diff(t, prepend=t[0])  # ns since previous record
         code = T[:, 2]

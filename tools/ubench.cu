@@ -199,8 +199,50 @@ int contention()
     return 0;
 }
 
+// dependent-load latency vs footprint (TLB reach): 4000 hops, each to a
+// random 128-B line of a buffer of the given size (device-side init)
+__global__ void k_tlb_init(int *buf, size_t lines, uint64_t seed)
+{
+    // buf[line*32] = next line index*32 of a random cycle: use an LCG walk
+    // over lines with a multiplier coprime to lines (full period for odd step)
+    size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x;
+    if (i >= lines) return;
+    const size_t a = 2862933555777941757ull % lines | 1;  // odd, coprime to 2^k
+    buf[i * 32] = (int)(((i * a + 12345) % lines));       // line index
+}
+__global__ void k_tlb_chase(const int *buf, int steps, long long *out, int *sink, size_t start)
+{
+    size_t p = start;
+    long long t0 = clock64();
+    for (int i = 0; i < steps; i++) p = (size_t)__ldcg(buf + p * 32);
+    long long t1 = clock64();
+    out[0] = t1 - t0;
+    sink[0] = (int)p;
+}
+static int tlb()
+{
+    long long *d_c; int *sink;
+    CK(cudaMalloc(&d_c, 64)); CK(cudaMalloc(&sink, 64));
+    for (size_t mb : {16, 64, 256, 1024, 2048, 4096, 8192}) {
+        size_t bytes = mb << 20, lines = bytes / 128;
+        int *d; CK(cudaMalloc(&d, bytes));
+        k_tlb_init<<<(unsigned)((lines + 255) / 256), 256>>>(d, lines, 1);
+        CK(cudaDeviceSynchronize());
+        long long hc = 0;
+        for (int rep = 0; rep < 2; rep++) {
+            k_tlb_chase<<<1, 1>>>(d, 4000, d_c, sink, (lines / 3) * rep + 7);
+            CK(cudaDeviceSynchronize());
+        }
+        CK(cudaMemcpy(&hc, d_c, 8, cudaMemcpyDeviceToHost));
+        printf("dependent ld.cg over %5zu MB (random lines): %.0f cycles/hop\n", mb, hc / 4000.0);
+        CK(cudaFree(d));
+    }
+    return 0;
+}
+
 int main(int argc, char **argv)
 {
+    if (argc > 1 && std::string(argv[1]) == "tlb") return tlb();
     if (argc > 1 && std::string(argv[1]) == "contention") return contention();
     if (argc > 1 && std::string(argv[1]) == "hotset") return hotset();
     int sms; CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0));
