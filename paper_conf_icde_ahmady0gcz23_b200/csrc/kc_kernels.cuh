@@ -246,7 +246,11 @@ __device__ __forceinline__ void probe(int tag, int64_t val)
     r[0] = blockIdx.x; r[1] = tag; r[2] = t; r[3] = val;
 }
 #define PROBE(tag, val) probe(tag, val)
+#ifdef KC_PROBE_W
+#define PROBE_W(tag, val) probe(tag, val)
+#else
 #define PROBE_W(tag, val) ((void)0)
+#endif
 #else
 #define PROBE_W(tag, val) ((void)0)
 #define PROBE(tag, val) ((void)0)
@@ -542,15 +546,17 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u
 {
     const int wib = threadIdx.x >> 5;
     const int uu[4] = {u0, u1, u2, u3};
-    bool won[4];
-#pragma unroll
-    for (int r = 0; r < 4; r++) won[r] = ((hm >> r) & 1u) && claim(A, uu[r]);
+    // row bounds and claims issued together (independent round trips)
     int64_t b0[4], b1[4];
 #pragma unroll
     for (int r = 0; r < 4; r++) {
-        b0[r] = won[r] ? ld_ro_i64(A.rowptr + uu[r]) : 0;
-        b1[r] = won[r] ? ld_ro_i64(A.rowptr + uu[r] + 1) : 0;
+        const bool h = (hm >> r) & 1u;
+        b0[r] = h ? ld_ro_i64(A.rowptr + uu[r]) : 0;
+        b1[r] = h ? ld_ro_i64(A.rowptr + uu[r] + 1) : 0;
     }
+    bool won[4];
+#pragma unroll
+    for (int r = 0; r < 4; r++) won[r] = ((hm >> r) & 1u) && claim(A, uu[r]);
 #pragma unroll
     for (int r = 0; r < 4; r++) {
         if (won[r] && b1[r] > b0[r]) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[r]));
@@ -620,6 +626,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
         // while this batch's deg loads and atomics (L2) complete
         int32_t un[kUnroll];
         if (a < limit) gather(a, un);
+        if (LOCAL && threadIdx.x == 0) PROBE_W(51, un[0]);
         while (a < limit) {
             int32_t u[kUnroll];
 #pragma unroll
@@ -634,9 +641,11 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             int32_t d[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) d[r] = u[r] >= 0 ? ld_cg_i32(A.deg + u[r]) : -1;
+            if (LOCAL && threadIdx.x == 0) PROBE_W(52, d[0]);
             int old[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
+            if (LOCAL && threadIdx.x == 0) PROBE_W(53, old[0]);
             unsigned hm = 0;
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
@@ -646,7 +655,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             }
             if (LOCAL && threadIdx.x == 0) PROBE_W(12, a);
             if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, gcnt);
-            if (LOCAL && threadIdx.x == 0) PROBE_W(13, __popc(hm));
+            if (LOCAL && threadIdx.x == 0) PROBE_W(54, __popc(hm));
             a = an;
         }
         a = limit;
@@ -683,6 +692,7 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         if (subs) { *subs += 1; *tmax = max(*tmax, T); }
         if (threadIdx.x == 0) PROBE(3, sm.lcnt[nx]);
         __syncthreads();
+        if (threadIdx.x == 0) PROBE(4, 0);
         if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
         cur = nx;
     }
@@ -1056,6 +1066,12 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         } else {
             c.st_hubarcs += c.ae - c.as;
         }
+        if (removed >= p.n) {  // every vertex claimed: the rest of the level changes nothing
+            if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
+            c.phase = PH_DONE;
+            c.solo = 0;
+            return;
+        }
         if (gcnt > c.gq_cnt) {  // hub / overflow vertices pending: HUB phase
             c.phase = PH_HUB;
             c.s = c.gq_cnt; c.e = gcnt; c.as = c.gq_arc; c.ae = garc;
@@ -1138,12 +1154,15 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
     if (threadIdx.x == 0) {
         State *S = A.S;
         PROBE(33, 0);
-        const uint32_t gen = ld_acquire_u32(&S->bar_gen);
-        const uint32_t t = atom_add_release_u32(&S->bar_count, 1u);
+        // bar_count is monotone and every barrier adds gridDim.x, so the
+        // generation follows from the ticket: one round trip to arrive.  The
+        // acq_rel RMW chain on bar_count orders every CTA's counter updates
+        // before the last arriver's snapshot (no separate fence).
+        const uint32_t t = atom_add_acq_rel_u32(&S->bar_count, 1u);
+        const uint32_t gen = t / (uint32_t)gridDim.x;
         PROBE(35, t);
         Snap sn;
         if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
-            __threadfence();
             sn = take_snapshot(S, gridDim.x);
             S->snap[(gen + 1u) & 1u] = sn;
             st_release_u32(&S->bar_gen, gen + 1u);

