@@ -193,7 +193,7 @@ struct Smem {
     unsigned long long scan_q[kWarps];
     unsigned long long tot_q, base_o, base_k;
     int32_t red_min[kWarps];
-    int64_t bloom_level;
+    int64_t bloom_level;  // alive-list length the filter was built from
     int32_t bloom_on;
     int32_t pool_on;             // this phase uses the work pool (grid-uniform)
     int32_t pool_done;           // pool drained (set by any warp of this CTA)
@@ -591,6 +591,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
     }
     int64_t i = lo;
     int64_t a = a0;
+    if (!LOCAL && threadIdx.x == 0) PROBE_W(60, a1 - a0);
     if (LOCAL && threadIdx.x == 0) PROBE_W(10, a1 - a0);
     while (a < a1) {
         const int64_t j = i + lane;
@@ -817,16 +818,23 @@ __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0) { sm.bloom_level = c.level; sm.bloom_on = 1; }
+    if (threadIdx.x == 0) { sm.bloom_level = c.src_len; sm.bloom_on = 1; }
     __syncthreads();
 }
 
-// Decide (CTA-uniform) whether walking `arcs` arcs this phase pays for a filter.
+// Decide (CTA-uniform) whether this phase's walks use the filter.  The alive
+// set only shrinks, so a filter built at an earlier level stays a valid
+// superset test; it is rebuilt once the alive list has halved since (fewer
+// false positives).  Dead targets then cost a shared-memory probe instead of
+// a scattered L2/HBM request -- the per-SM request rate is what bounds a
+// cascade walked by one CTA.
 __device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &sm, int64_t arcs)
 {
-    if (!A.S->prm.bloom || c.src_sel < 0 || c.src_len > kBloomMaxA) return false;
-    if (sm.bloom_on && sm.bloom_level == c.level) return true;
-    if (arcs < 4 * c.src_len + 65536) return false;
+    (void)arcs;
+    if (!A.S->prm.bloom) return false;
+    const bool have = sm.bloom_on != 0;
+    if (have && c.src_len * 2 > sm.bloom_level) return true;
+    if (c.src_sel < 0 || c.src_len > kBloomMaxA) return have;
     bloom_build(A, c, sm);
     return true;
 }
