@@ -28,8 +28,9 @@
  *             inputs are made undirected by ignoring direction, reading R2).
  *             These preconditions are NOT checked on the fast path; call
  *             kcore_validate_csr() (tests/debug) to check them.
- *  - core_out: int32[n] output; it also serves as the degree work array
- *             (deg[] becomes core[] in place).
+ *  - core_out: int32[n] output.  core_out[v] is written once, when v is
+ *             removed at level k (the removal level is the core
+ *             number); the working degrees live in the workspace.
  *  - Ownership: the caller owns all inputs/outputs; inputs are never
  *             modified; the library never frees caller memory.  Scratch
  *             (kcore_workspace_size bytes) is either caller-provided via
@@ -64,9 +65,6 @@ typedef enum {
 
 /* kcore_options.flags */
 #define KCORE_FLAG_NO_BLOOM 1   /* disable the shared-memory alive-set filter (ablation) */
-#define KCORE_FLAG_POOL 2       /* in-phase work pool: vertices too big for one CTA are   */
-                                /* split into items any idle warp takes in the same phase */
-                                /* (experimental; default off -- DESIGN.md)               */
 
 /* Algorithms selectable through kcore_options.algo. */
 #define KCORE_ALGO_PERSISTENT 0 /* default: one persistent kernel, device-resident loop */

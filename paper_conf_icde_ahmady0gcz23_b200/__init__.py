@@ -35,7 +35,6 @@ KCORE_EUNSUPPORTED = -6
 ALGO_PERSISTENT = 0
 ALGO_HOSTLOOP = 1
 FLAG_NO_BLOOM = 1
-FLAG_POOL = 2
 
 # every symbol include/kcore.h declares (checked by tests/test_abi.py)
 EXPORTS = (
@@ -169,7 +168,7 @@ def _check_csr_tensors(rowptr, colidx):
 
 def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=None,
                     algo: int = ALGO_PERSISTENT, blocks_per_sm: int = 0, solo_arcs: int = 0,
-                    solo_scan: int = 0, bloom: bool = True, pool: bool = False, trace=None,
+                    solo_scan: int = 0, bloom: bool = True, trace=None,
                     trace_cta=None, stats: bool = False):
     """Core numbers of the graph (rowptr int64[n+1], colidx int32[m] CUDA tensors).
 
@@ -188,7 +187,7 @@ def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=
                    workspace.numel() * workspace.element_size() if workspace is not None else 0,
                    trace.data_ptr() if trace is not None else None,
                    trace.shape[0] if trace is not None else 0,
-                   (0 if bloom else FLAG_NO_BLOOM) | (FLAG_POOL if pool else 0), 0,
+                   (0 if bloom else FLAG_NO_BLOOM), 0,
                    trace_cta.data_ptr() if trace_cta is not None else None)
     st = _Stats()
     with torch.cuda.device(dev):

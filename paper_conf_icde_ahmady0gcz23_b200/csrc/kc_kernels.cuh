@@ -82,21 +82,20 @@ constexpr int kBloomMaxA = KC_BLOOM_MAXA;  // build only for alive lists up to t
 constexpr int kUnroll = 4;  // arcs per lane in flight per batch (handle_hits assumes 4)
 constexpr int kBatch = 32 * kUnroll;
 constexpr int kTraceFields = 8;
-// Work pool: vertices too big for one CTA are split into items of about
-// kItemArcs arcs that any idle warp of the grid takes within the same phase.
-#ifndef KC_POOL_CAP
-#define KC_POOL_CAP (1 << 16)
+// With the alive-set filter on (most removed targets never reach L2), walks
+// may skip the deg pre-read and decrement every target that passes it: one
+// scattered atomic instead of a read followed by an atomic on the same line.
+// Removed targets then take garbage decrements -- harmless, their core was
+// written when they were claimed (deg is a private working array).
+#ifndef KC_AO_HUB
+#define KC_AO_HUB 1
 #endif
-constexpr int kPoolCap = KC_POOL_CAP;  // items per phase (beyond: global queue)
-#ifndef KC_ITEM
-#define KC_ITEM 256
+#ifndef KC_AO_LOCAL
+#define KC_AO_LOCAL 1
 #endif
-constexpr int kItemArcs = KC_ITEM;
-constexpr int kItemMax = 64;          // items per vertex at most
-constexpr int kItemLenBits = 26;      // item word: ((beg + 1) << 26) | len
-constexpr unsigned long long kItemNull = 1ULL;  // a reserved slot left unused
-static_assert(kItemArcs >= kItemMax, "every item of a split vertex must be non-empty");
-
+#ifndef KC_AO_ALWAYS
+#define KC_AO_ALWAYS 0
+#endif
 enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
 struct Ctrl {
@@ -132,7 +131,7 @@ struct Params {
     int32_t solo_arcs;  // HUB phases with <= this many arcs run solo
     int32_t solo_scan;  // LEVEL phases over <= this many entries run solo
     int32_t bloom;      // 0 disables the Bloom filter
-    int32_t pool;       // 0 disables the work pool
+    int32_t pad;
 };
 
 struct State {
@@ -144,8 +143,6 @@ struct State {
     alignas(128) uint32_t bar_gen;              // grid barrier generation
     Snap snap[2];                               // counters at barrier gen, by gen & 1
     alignas(128) unsigned long long arcs_walked;
-    alignas(128) unsigned long long pool_pk;    // packed (items reserved << 32) | pending units
-    alignas(128) unsigned long long pool_head;  // next ticket
     alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
     alignas(128) Params prm;
     int64_t *trace;                             // optional [trace_cap][kTraceFields]
@@ -157,7 +154,8 @@ struct State {
 struct KArgs {
     const int64_t *rowptr;
     const int32_t *colidx;
-    int32_t *deg;       // == core_out
+    int32_t *deg;       // working degrees (workspace): only decrease, garbage once removed
+    int32_t *core;      // core_out: written once per vertex, when it is claimed at level k
     int32_t *order;     // removal order (all vertices)
     uint32_t *claimed;  // claim bit per vertex
     int32_t *gq_v;      // global queue: vertex, row begin, arc prefix
@@ -167,8 +165,6 @@ struct KArgs {
     int32_t *seg_len[2];  // entries of segment b in alive[x]: seg_len[x][b]
     int64_t seg_R;        // segment region size: segment b lives at [b*R, b*R + len)
     int32_t nseg;         // = persistent grid size
-    int32_t pool_on;      // 1: grid phases use the work pool (persistent kernel only)
-    unsigned long long *pool;  // [kPoolCap] item words, 0 = empty
     State *S;
     int64_t n;
 };
@@ -195,10 +191,6 @@ struct Smem {
     int32_t red_min[kWarps];
     int64_t bloom_level;  // alive-list length the filter was built from
     int32_t bloom_on;
-    int32_t pool_on;             // this phase uses the work pool (grid-uniform)
-    int32_t pool_done;           // pool drained (set by any warp of this CTA)
-    int32_t pad3;
-    unsigned long long pool_arcs;  // arcs walked from pool items by this CTA this phase
     Ctrl ctrl;
     Snap snap;
     uint32_t bloom[kBloomWords];
@@ -396,70 +388,6 @@ __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gc
     gcnt = 0;
 }
 
-__device__ __forceinline__ void st_relaxed_u64(unsigned long long *p, unsigned long long v)
-{
-    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-
-// Push the vertices of the lanes where `want` into the work pool, each split
-// into ceil(d / kItemArcs) items (at most kItemMax).  One packed atomic
-// reserves the slots and adds them to the pending count before any item is
-// visible.  Returns true for lanes whose vertex did not fit (pool full for
-// this phase): the caller sends those to the global queue.
-__device__ __noinline__ bool pool_push(const KArgs &A, bool want, int32_t dv, int64_t bv)
-{
-    const int lane = threadIdx.x & 31;
-    if (__ballot_sync(kFull, want) == 0) return false;
-    int nj = 0;
-    if (want) nj = min((dv + kItemArcs - 1) / kItemArcs, kItemMax);
-    int incl = nj;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int t = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += t;
-    }
-    const int tot = __shfl_sync(kFull, incl, 31);
-    const int ex = incl - nj;
-    unsigned long long base = 0;
-    int ok = 0;
-    if (lane == 0) {
-        const unsigned long long old =
-            atomicAdd(&A.S->pool_pk, ((unsigned long long)tot << 32) | (unsigned long long)tot);
-        base = old >> 32;
-        PROBE(20, (int64_t)((base << 16) | (unsigned long long)tot));
-        if (base + (unsigned long long)tot <= (unsigned long long)kPoolCap) ok = 1;
-        else atomicAdd(&A.S->pool_pk, 0ULL - (unsigned long long)tot);  // not pending after all
-        __threadfence();
-    }
-    base = __shfl_sync(kFull, base, 0);
-    ok = __shfl_sync(kFull, ok, 0);
-    for (int x0 = 0; x0 < tot; x0 += 32) {
-        const int x = x0 + lane;
-        int pos = 0;
-#pragma unroll
-        for (int bs = 16; bs >= 1; bs >>= 1) {
-            const int q = __shfl_sync(kFull, ex, pos + bs);
-            if (q <= x) pos += bs;
-        }
-        const int njo = __shfl_sync(kFull, nj, pos);
-        const int dvo = __shfl_sync(kFull, dv, pos);
-        const int exo = __shfl_sync(kFull, ex, pos);
-        const int64_t bvo = __shfl_sync(kFull, bv, pos);
-        if (x < tot && base + (unsigned long long)x < (unsigned long long)kPoolCap) {
-            unsigned long long word = kItemNull;
-            if (ok) {
-                const int per = (dvo + njo - 1) / njo;
-                const int ib = (x - exo) * per;
-                const int il = min(per, dvo - ib);
-                word = ((unsigned long long)(bvo + ib + 1) << kItemLenBits) | (unsigned long long)il;
-            }
-            st_relaxed_u64(A.pool + base + x, word);
-        }
-    }
-    __syncwarp();
-    return want && !ok;
-}
-
 // Route claimed vertices (one per lane where `won`): reserve their slots in
 // the removal order right away (a vertex is claimed only after every vertex
 // whose processing made it reach k was claimed, so claim-time slots form a
@@ -516,7 +444,6 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
             tog = true;
         }
     }
-    if (sm.pool_on) tog = pool_push(A, tog, dv, bv);
     const unsigned bg = __ballot_sync(kFull, tog);
     if (bg) {
         const int c = __popc(bg);
@@ -541,7 +468,7 @@ __device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
 // --------------------------------------------------------- arc walking
 // Hits of one batch (u reached k): claim, fetch row bounds, prefetch the
 // row's first line for the next hop, route.  Out of line: rare path.
-__device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u0, int u1, int u2, int u3,
+__device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int k, int nx, int u0, int u1, int u2, int u3,
                                          unsigned hm, int &gcnt)
 {
     const int wib = threadIdx.x >> 5;
@@ -558,6 +485,9 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u
 #pragma unroll
     for (int r = 0; r < 4; r++) won[r] = ((hm >> r) & 1u) && claim(A, uu[r]);
 #pragma unroll
+    for (int r = 0; r < 4; r++)
+        if (won[r]) A.core[uu[r]] = k;
+#pragma unroll
     for (int r = 0; r < 4; r++) {
         if (won[r] && b1[r] > b0[r]) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[r]));
         route_won(A, sm, wib, won[r], uu[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, gcnt);
@@ -573,7 +503,7 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int nx, int u
 template <bool LOCAL>
 __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, const int cur, const int nx,
                                      int64_t s, int64_t e, int64_t ae, int64_t a0, int64_t a1,
-                                     bool use_bloom, int &lmin, int &gcnt)
+                                     bool use_bloom, bool atom_only, int &lmin, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
     // first entry: largest i in [s,e) with P(i) <= a0 (32-ary search)
@@ -591,8 +521,6 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
     }
     int64_t i = lo;
     int64_t a = a0;
-    if (!LOCAL && threadIdx.x == 0) PROBE_W(60, a1 - a0);
-    if (LOCAL && threadIdx.x == 0) PROBE_W(10, a1 - a0);
     while (a < a1) {
         const int64_t j = i + lane;
         int64_t wq = LLONG_MAX, wbeg = 0;
@@ -627,7 +555,6 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
         // while this batch's deg loads and atomics (L2) complete
         int32_t un[kUnroll];
         if (a < limit) gather(a, un);
-        if (LOCAL && threadIdx.x == 0) PROBE_W(51, un[0]);
         while (a < limit) {
             int32_t u[kUnroll];
 #pragma unroll
@@ -641,22 +568,18 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             }
             int32_t d[kUnroll];
 #pragma unroll
-            for (int r = 0; r < kUnroll; r++) d[r] = u[r] >= 0 ? ld_cg_i32(A.deg + u[r]) : -1;
-            if (LOCAL && threadIdx.x == 0) PROBE_W(52, d[0]);
+            for (int r = 0; r < kUnroll; r++)
+                d[r] = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_cg_i32(A.deg + u[r]));
             int old[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
-            if (LOCAL && threadIdx.x == 0) PROBE_W(53, old[0]);
             unsigned hm = 0;
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
                 if (old[r] == k + 1) hm |= 1u << r;
-                else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
                 else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
             }
-            if (LOCAL && threadIdx.x == 0) PROBE_W(12, a);
-            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, nx, u[0], u[1], u[2], u[3], hm, gcnt);
-            if (LOCAL && threadIdx.x == 0) PROBE_W(54, __popc(hm));
+            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, k, nx, u[0], u[1], u[2], u[3], hm, gcnt);
             a = an;
         }
         a = limit;
@@ -666,7 +589,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
 
 // Drain this CTA's local frontier (list `cur`) breadth-first with CTA-local
 // sub-rounds.  Returns the number of arcs walked.
-__device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, bool use_bloom,
+__device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, bool use_bloom, bool atom_only,
                                int &lmin, int &gcnt, int64_t *subs = nullptr, int64_t *tmax = nullptr)
 {
     const int wib = threadIdx.x >> 5;
@@ -688,7 +611,7 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         int64_t C = (T + kWarps - 1) / kWarps;
         C = ((C + kBatch - 1) / kBatch) * kBatch;
         const int64_t a0 = (int64_t)wib * C;
-        if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, lmin, gcnt);
+        if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, atom_only, lmin, gcnt);
         walked += T;
         if (subs) { *subs += 1; *tmax = max(*tmax, T); }
         if (threadIdx.x == 0) PROBE(3, sm.lcnt[nx]);
@@ -698,97 +621,6 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         cur = nx;
     }
     return walked;
-}
-
-// One pool item: arcs [beg, beg+len) walked by one warp; hits go back to
-// the pool (or the global queue when it is full).
-__device__ __forceinline__ void walk_item(const KArgs &A, Smem &sm, const int k, int64_t beg, int len,
-                                          int &lmin, int &gcnt)
-{
-    const int lane = threadIdx.x & 31;
-    for (int a = 0; a < len; a += kBatch) {
-        int32_t u[kUnroll];
-#pragma unroll
-        for (int r = 0; r < kUnroll; r++) {
-            const int x = a + r * 32 + lane;
-            u[r] = x < len ? ld_stream_i32(A.colidx + beg + x) : -1;
-        }
-        int32_t d[kUnroll];
-#pragma unroll
-        for (int r = 0; r < kUnroll; r++) d[r] = u[r] >= 0 ? ld_cg_i32(A.deg + u[r]) : -1;
-        int old[kUnroll];
-#pragma unroll
-        for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
-        unsigned hm = 0;
-#pragma unroll
-        for (int r = 0; r < kUnroll; r++) {
-            if (old[r] == k + 1) hm |= 1u << r;
-            else if (old[r] != INT_MIN && old[r] <= k) atomicAdd(A.deg + u[r], 1);
-            else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
-        }
-        if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, -1, u[0], u[1], u[2], u[3], hm, gcnt);
-    }
-}
-
-// Take pool items until the phase's pending count (one unit per CTA until
-// its own scan + local drain is done, plus one per pushed item until it is
-// walked) reaches zero.  Each warp holds one ticket = one slot; lane 0 polls
-// the slot and, every few polls, the pending count.
-__device__ void pool_consume(const KArgs &A, Smem &sm, const int k, int &lmin, int &gcnt)
-{
-    const int lane = threadIdx.x & 31;
-    State *S = A.S;
-    volatile int32_t *done = &sm.pool_done;
-    unsigned long long walked = 0;
-    while (true) {
-        unsigned long long w = 0;
-        if (lane == 0) {
-            const unsigned long long t = atomicAdd(&S->pool_head, 1ULL);
-            unsigned spins = 0;
-            while (true) {
-                if (t < (unsigned long long)kPoolCap) {
-                    w = ld_relaxed_u64(A.pool + t);
-                    if (w) break;
-                }
-                if (*done) break;
-                if ((++spins & 3u) == 0u && (uint32_t)ld_relaxed_u64(&S->pool_pk) == 0u) {
-                    *done = 1;
-                    break;
-                }
-                __nanosleep(64);
-            }
-            if (w) { st_relaxed_u64(A.pool + t, 0ULL); PROBE(21, (int64_t)t); }
-            else if (threadIdx.x == 0) PROBE(23, (int64_t)t);
-        }
-        w = __shfl_sync(kFull, w, 0);
-        if (w == 0) break;
-        if (w == kItemNull) continue;
-        const int64_t beg = (int64_t)(w >> kItemLenBits) - 1;
-        const int len = (int)(w & ((1ULL << kItemLenBits) - 1ULL));
-        walk_item(A, sm, k, beg, len, lmin, gcnt);
-        walked += (unsigned long long)len;
-        __syncwarp();
-        if (lane == 0) { atomicAdd(&S->pool_pk, ~0ULL); PROBE(22, len); }  // after this item's pushes
-    }
-    if (lane == 0 && walked) atomicAdd(&sm.pool_arcs, walked);
-}
-
-// The CTA's own unit is released once its scan / queue walk and local drain
-// are done (its pushes are already counted); then every warp takes items.
-__device__ __forceinline__ void pool_phase_tail(const KArgs &A, const Ctrl &c, Smem &sm, int &lmin, int &gcnt)
-{
-    const int wib = threadIdx.x >> 5;
-    if (!sm.pool_on) return;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        __threadfence();
-        atomicAdd(&A.S->pool_pk, ~0ULL);
-        PROBE(31, 0);
-    }
-    pool_consume(A, sm, c.k, lmin, gcnt);
-    gq_flush(A, sm, wib, gcnt);
-    __syncthreads();
-    if (threadIdx.x == 0) PROBE(32, 0);
 }
 
 // Bloom filter of the alive list at level start (built once per level).
@@ -899,6 +731,9 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
             for (int j = 0; j < kScanItems; j++)
                 if ((km >> j) & 1u) dst[pos++] = vv[j];
         }
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++)
+            if ((wm >> j) & 1u) A.core[vv[j]] = k;
         if (__any_sync(kFull, wm != 0)) {
             // row bounds of every claimed vertex first (all loads in flight), then route
             int64_t b0[kScanItems];
@@ -972,24 +807,21 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.bud_hub = c.light ? kHubLight : kHubHeavy;
         sm.bud_sub = c.light ? kSubLight : kSubHeavy;
         sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
-        sm.pool_on = (A.pool_on && nblk > 1) ? 1 : 0;
-        sm.pool_done = 0;
-        sm.pool_arcs = 0ULL;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
     __syncthreads();
     cta_time(A, c, 1);
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
+    const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_LOCAL;
     int64_t subs = 0, tmax = 0;
-    const int64_t walked = local_drain(A, sm, c.k, 0, bl, lmin, gcnt, &subs, &tmax);
+    const int64_t walked = local_drain(A, sm, c.k, 0, bl, ao, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
-    pool_phase_tail(A, c, sm, lmin, gcnt);
     __syncthreads();
-    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked + (int64_t)sm.pool_arcs); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
+    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
     if (threadIdx.x == 0) {
-        const unsigned long long wk = (unsigned long long)walked + sm.pool_arcs;
+        const unsigned long long wk = (unsigned long long)walked;
         if (wk) atomicAdd(&A.S->arcs_walked, wk);
         if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
     }
@@ -1017,28 +849,25 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
         sm.bud_hub = c.light ? kHubLight : kHubHeavy;
         sm.bud_sub = c.light ? kSubLight : kSubHeavy;
         sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
-        sm.pool_on = (A.pool_on && nblk > 1) ? 1 : 0;
-        sm.pool_done = 0;
-        sm.pool_arcs = 0ULL;
     }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
     const bool bl = want_bloom(A, c, sm, cta_arcs);
+    const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_HUB;
     const int64_t a0 = c.as + gw * C;
     if (a0 < c.ae)
-        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, lmin, gcnt);
+        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt);
     int64_t walked = cta_arcs;
     __syncthreads();
     cta_time(A, c, 1);
     int64_t subs = 0, tmax = 0;
-    walked += local_drain(A, sm, c.k, 0, bl, lmin, gcnt, &subs, &tmax);
+    walked += local_drain(A, sm, c.k, 0, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
-    pool_phase_tail(A, c, sm, lmin, gcnt);
     __syncthreads();
-    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked + (int64_t)sm.pool_arcs); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
+    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
     if (threadIdx.x == 0) {
-        const unsigned long long wk = (unsigned long long)walked + sm.pool_arcs;
+        const unsigned long long wk = (unsigned long long)walked;
         if (wk) atomicAdd(&A.S->arcs_walked, wk);
         if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
     }
@@ -1132,8 +961,6 @@ __device__ __forceinline__ Snap take_snapshot(State *S, unsigned grid)
     sn.pad = 0;
     S->alive_out = 0ULL;
     S->min_next = INT_MAX;
-    S->pool_pk = (unsigned long long)grid;  // one pending unit per CTA
-    S->pool_head = 0ULL;
     return sn;
 }
 
@@ -1318,8 +1145,6 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
         S->bar_count = 0u;
         S->bar_gen = 0u;
         S->arcs_walked = 0ULL;
-        S->pool_pk = 0ULL;
-        S->pool_head = 0ULL;
         Ctrl z;
         init_ctrl(z);
         S->pub = z;

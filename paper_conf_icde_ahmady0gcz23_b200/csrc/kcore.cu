@@ -66,7 +66,7 @@ struct Carve {
     int64_t *gq_beg, *gq_arc;
     int32_t *alive0, *alive1;
     int32_t *seg0, *seg1;
-    unsigned long long *pool;
+    int32_t *deg;
 };
 
 constexpr int kMaxSeg = 16384;  // one alive-list segment per warp of the persistent grid
@@ -91,7 +91,7 @@ size_t carve(void *base, int64_t n, Carve *c)
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     t.seg1 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
-    t.pool = (unsigned long long *)take(sizeof(unsigned long long) * kPoolCap);
+    t.deg = (int32_t *)take(sizeof(int32_t) * nn);
     if (c) *c = t;
     return off;
 }
@@ -209,7 +209,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     carve(ws, n, &cv);
     A.rowptr = rowptr;
     A.colidx = colidx;
-    A.deg = core_out;
+    A.deg = cv.deg;
+    A.core = core_out;
     A.order = (opt && opt->order_out) ? cv.order : nullptr;  // record the peel order only on request
     A.claimed = cv.claimed;
     A.gq_v = cv.gq_v;
@@ -221,8 +222,6 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.seg_len[1] = cv.seg1;
     A.nseg = grid;
     A.seg_R = (n + A.nseg - 1) / A.nseg;
-    A.pool = cv.pool;
-    A.pool_on = (algo == KCORE_ALGO_PERSISTENT && opt && (opt->flags & KCORE_FLAG_POOL)) ? 1 : 0;
     A.S = cv.S;
     A.n = n;
 
@@ -230,7 +229,6 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaEventCreate(&ev0));
         KC_CUDA(cudaEventCreate(&ev1));
     }
-    KC_CUDA(cudaMemsetAsync(cv.pool, 0, sizeof(unsigned long long) * kPoolCap, st));
     k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, trace,
                                    trace ? opt->trace_cta_out : nullptr, trace_cap);
     KC_CUDA(cudaGetLastError());

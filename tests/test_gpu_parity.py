@@ -40,7 +40,7 @@ def _check(rp, ci, ref=None, **kw):
 
 
 VARIANTS = [dict(), dict(solo_arcs=16384, solo_scan=32768), dict(bloom=False), dict(algo=kc.ALGO_HOSTLOOP),
-            dict(solo_arcs=1 << 30, solo_scan=1 << 30), dict(pool=True)]
+            dict(solo_arcs=1 << 30, solo_scan=1 << 30)]
 
 
 # ------------------------------------------------------------ paper pins

@@ -26,6 +26,16 @@ __global__ void k_walk(const int *colidx, int *deg, long long chunks_per_warp, i
             int d[U];
 #pragma unroll
             for (int r = 0; r < U; r++) d[r] = __ldcg(deg + u[r]);
+            if (MODE == 3) {  // red.sub without return, no deg read
+#pragma unroll
+                for (int r = 0; r < U; r++) atomicSub(deg + u[r], 1);
+                continue;
+            }
+            if (MODE == 4) {  // atomicSub with return, no deg read
+#pragma unroll
+                for (int r = 0; r < U; r++) acc += atomicSub(deg + u[r], 1);
+                continue;
+            }
             if (MODE == 1) {
 #pragma unroll
                 for (int r = 0; r < U; r++) if (d[r] > K) acc += atomicSub(deg + u[r], 1);
@@ -63,6 +73,19 @@ int main()
     std::vector<int> hd(N, 1 << 30);
     CK(cudaMemcpy(deg, hd.data(), (size_t)N * 4, cudaMemcpyHostToDevice));
     const int block = 768, warps = block / 32;
+    for (int hot : {1 << 22, 1 << 16, 1 << 12}) {
+        std::vector<int> hh(M);
+        for (long long i = 0; i < M; i++) hh[i] = h[i] % hot;
+        CK(cudaMemcpy(ci, hh.data(), M * 4, cudaMemcpyHostToDevice));
+        const int grid = 148; const long long cpw = 32;
+        const double arcs = (double)grid * warps * cpw * 256;
+        float t;
+        t = run<4, 0>(ci, deg, grid, block, cpw, 0, sink); printf("hot %8d  ld only      : %8.1f G arcs/s\n", hot, arcs / (t * 1e6));
+        t = run<4, 1>(ci, deg, grid, block, cpw, 0, sink); printf("hot %8d  ld + atom    : %8.1f G arcs/s\n", hot, arcs / (t * 1e6));
+        t = run<4, 4>(ci, deg, grid, block, cpw, 0, sink); printf("hot %8d  atom (ret)   : %8.1f G arcs/s\n", hot, arcs / (t * 1e6));
+        t = run<4, 3>(ci, deg, grid, block, cpw, 0, sink); printf("hot %8d  red (no ret) : %8.1f G arcs/s\n", hot, arcs / (t * 1e6));
+    }
+    CK(cudaMemcpy(ci, h.data(), M * 4, cudaMemcpyHostToDevice));
     for (int grid : {1, 8, 148}) {
         const long long cpw = (grid == 148) ? 32 : 64;
         const double arcs = (double)grid * warps * cpw * 256;
