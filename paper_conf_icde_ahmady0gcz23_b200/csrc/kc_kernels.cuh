@@ -94,7 +94,7 @@ constexpr int kTraceFields = 8;
 #define KC_AO_LOCAL 1
 #endif
 #ifndef KC_AO_ALWAYS
-#define KC_AO_ALWAYS 0
+#define KC_AO_ALWAYS 1
 #endif
 enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
@@ -677,12 +677,20 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
     int lmin = INT_MAX;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    for (int64_t v = tid; v < A.n; v += stride) {
-        const int32_t d = (int32_t)(ld_ro_i64(A.rowptr + v + 1) - ld_ro_i64(A.rowptr + v));
-        A.deg[v] = d;
-        lmin = min(lmin, d);
+    // claim bits start set exactly for the isolated vertices (removed at
+    // k = 0 without a claim): a warp covers 32 consecutive, aligned ids
+    static_assert(kBlock % 32 == 0, "warps cover aligned 32-vertex words");
+    for (int64_t v0 = tid - (threadIdx.x & 31); v0 < A.n; v0 += stride) {
+        const int64_t v = v0 + (threadIdx.x & 31);
+        int32_t d = -1;
+        if (v < A.n) {
+            d = (int32_t)(ld_ro_i64(A.rowptr + v + 1) - ld_ro_i64(A.rowptr + v));
+            A.deg[v] = d;
+            lmin = min(lmin, d);
+        }
+        const unsigned iso = __ballot_sync(kFull, d == 0);
+        if ((threadIdx.x & 31) == 0) A.claimed[v0 >> 5] = iso;
     }
-    for (int64_t w = tid; w < (A.n + 31) / 32; w += stride) A.claimed[w] = 0u;
     if (threadIdx.x == 0) { sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
@@ -712,8 +720,14 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
         unsigned wm = 0, km = 0;
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
-            // at k = 0 the frontier is the isolated vertices: nothing can race for them
-            if (dd[j] == k) { if (k == 0 || claim(A, vv[j])) wm |= 1u << j; }
+            // deg <= k: v is in the k-shell.  Every alive vertex has deg >= k at
+            // level start; atomic-only walks may already have taken a
+            // not-yet-scanned k-shell vertex below k (its crossing to k+1 was
+            // before this level, so no peel claims it).  Removed vertices left
+            // in a lazily compacted list fail the claim.  At k = 0 the frontier
+            // is the isolated vertices: nothing walks, nothing races.
+            if (vv[j] < 0) continue;
+            if (dd[j] <= k) { if (k == 0 || claim(A, vv[j])) wm |= 1u << j; }
             else if (dd[j] > k) { lmin = min(lmin, dd[j]); km |= 1u << j; }
         }
         if (dst) {
