@@ -65,6 +65,12 @@ typedef enum {
 
 /* kcore_options.flags */
 #define KCORE_FLAG_NO_BLOOM 1   /* disable the shared-memory alive-set filter (ablation) */
+#define KCORE_FLAG_NO_L2_PERSIST 2 /* do not pin the working degrees in L2 (ablation).  By    */
+                                /* default the call launches with a persisting L2 access- */
+                                /* policy window over its claim bits + working degrees,   */
+                                /* raising cudaLimitPersistingL2CacheSize (device-wide,   */
+                                /* never lowered) to the window size if it is smaller, and */
+                                /* returns the lines to normal priority after the kernel. */
 
 /* Algorithms selectable through kcore_options.algo. */
 #define KCORE_ALGO_PERSISTENT 0 /* default: one persistent kernel, device-resident loop */

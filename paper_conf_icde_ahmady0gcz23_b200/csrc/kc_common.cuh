@@ -82,9 +82,74 @@ __device__ __forceinline__ int32_t ld_stream_i32(const int32_t *p)
 
 __device__ __forceinline__ int64_t ld_ro_i64(const int64_t *p) { return __ldg(p); }
 
+// L2 residency of the scattered working set (deg, claim bits): the 4 GB
+// adjacency stream of a big level must not evict it, or every scattered
+// atomic becomes an HBM read-modify-write.
+#ifndef KC_DEG_EVICT_LAST
+#define KC_DEG_EVICT_LAST 0
+#endif
+__device__ __forceinline__ uint64_t l2_evict_last_policy()
+{
+    uint64_t pol;
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ int32_t atom_dec_deg(int32_t *p, uint64_t pol)
+{
+#if KC_DEG_EVICT_LAST
+    int32_t old;
+    asm volatile("atom.global.L2::cache_hint.add.s32 %0, [%1], -1, %2;" : "=r"(old) : "l"(p), "l"(pol) : "memory");
+    return old;
+#else
+    (void)pol;
+    return atomicSub(p, 1);
+#endif
+}
+__device__ __forceinline__ int32_t ld_deg(const int32_t *p, uint64_t pol)
+{
+#if KC_DEG_EVICT_LAST
+    int32_t v;
+    asm volatile("ld.global.cg.L2::cache_hint.s32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+#else
+    (void)pol;
+    return __ldcg(p);
+#endif
+}
+__device__ __forceinline__ uint32_t atom_or_claim(uint32_t *p, uint32_t bit, uint64_t pol)
+{
+#if KC_DEG_EVICT_LAST
+    uint32_t old;
+    asm volatile("atom.global.L2::cache_hint.or.b32 %0, [%1], %2, %3;" : "=r"(old) : "l"(p), "r"(bit), "l"(pol) : "memory");
+    return old;
+#else
+    (void)pol;
+    return atomicOr(p, bit);
+#endif
+}
+
 // L2-coherent loads of data other CTAs write during the call (deg, queue)
 __device__ __forceinline__ int32_t ld_cg_i32(const int32_t *p) { return __ldcg(p); }
 __device__ __forceinline__ int64_t ld_cg_i64(const int64_t *p) { return __ldcg(p); }
+
+// Warm L2 with the adjacency row [b, e) of a vertex that was just claimed, so
+// the next hop's colidx gathers hit L2: one TMA bulk prefetch of the whole
+// row (16-byte aligned, capped at KC_BULK_PF bytes), or the first line only.
+#ifndef KC_BULK_PF
+#define KC_BULK_PF 0
+#endif
+__device__ __forceinline__ void prefetch_row(const int32_t *colidx, int64_t b, int64_t e)
+{
+#if KC_BULK_PF > 0
+    const uintptr_t lo = reinterpret_cast<uintptr_t>(colidx + b) & ~(uintptr_t)15;
+    uintptr_t hi = (reinterpret_cast<uintptr_t>(colidx + e) + 15) & ~(uintptr_t)15;
+    if (hi - lo > (uintptr_t)KC_BULK_PF) hi = lo + KC_BULK_PF;
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(lo), "r"((uint32_t)(hi - lo)) : "memory");
+#else
+    (void)e;
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(colidx + b));
+#endif
+}
 
 __device__ __forceinline__ unsigned lanemask_lt()
 {

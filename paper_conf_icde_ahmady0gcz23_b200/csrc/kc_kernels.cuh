@@ -87,6 +87,12 @@ constexpr int kTraceFields = 8;
 // scattered atomic instead of a read followed by an atomic on the same line.
 // Removed targets then take garbage decrements -- harmless, their core was
 // written when they were claimed (deg is a private working array).
+#ifndef KC_ROUTE4
+#define KC_ROUTE4 1
+#endif
+#ifndef KC_FASTSUB
+#define KC_FASTSUB 1
+#endif
 #ifndef KC_AO_HUB
 #define KC_AO_HUB 1
 #endif
@@ -459,10 +465,113 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
     __syncwarp();
 }
 
+// route_won for four candidates per lane (one batch of a walk or a scan step):
+// the same decisions as four route_won calls, with ONE order/removed update,
+// ONE budget reservation and one local-list reservation for the whole warp
+// (the shared-memory atomics are a dependent chain on the hit path).
+__device__ __noinline__ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int32_t v1,
+                                        int32_t v2, int32_t v3, int32_t d0, int32_t d1, int32_t d2, int32_t d3,
+                                        int64_t b0, int64_t b1, int64_t b2, int64_t b3, int nx, int &gcnt)
+{
+    const int lane = threadIdx.x & 31;
+    const unsigned lt = lanemask_lt();
+    const int32_t vv[4] = {v0, v1, v2, v3};
+    const int32_t dd[4] = {d0, d1, d2, d3};
+    const int64_t bb[4] = {b0, b1, b2, b3};
+    unsigned bal[4];
+    int off[4], tot = 0;
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        bal[r] = __ballot_sync(kFull, (wm >> r) & 1u);
+        off[r] = tot;
+        tot += __popc(bal[r]);
+    }
+    if (tot == 0) return;
+    if (A.order) {  // peel order requested: slots in claim order
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(&A.S->ord_tail, (unsigned long long)tot);
+        base = __shfl_sync(kFull, base, 0);
+#pragma unroll
+        for (int r = 0; r < 4; r++)
+            if ((wm >> r) & 1u) A.order[base + off[r] + __popc(bal[r] & lt)] = vv[r];
+    } else if (lane == 0) {
+        atomicAdd(&sm.removed, tot);
+    }
+    unsigned cm = 0;
+#pragma unroll
+    for (int r = 0; r < 4; r++)
+        if (((wm >> r) & 1u) && dd[r] > 0 && dd[r] <= sm.bud_hub && nx >= 0) cm |= 1u << r;
+    unsigned cb[4];
+    int coff[4], ctot = 0, sumd = 0;
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        cb[r] = __ballot_sync(kFull, (cm >> r) & 1u);
+        coff[r] = ctot;
+        ctot += __popc(cb[r]);
+        if ((cm >> r) & 1u) sumd += dd[r];
+    }
+    unsigned lm = 0;  // candidates that go to the local list
+    int lbase = 0;
+    if (ctot) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sumd += __shfl_xor_sync(kFull, sumd, o);
+        int ok = 0;
+        if (lane == 0) {
+            const int oa = atomicAdd(&sm.larc[nx], sumd);
+            if (oa + sumd <= sm.bud_sub) {
+                const int op = atomicAdd(&sm.lphase, sumd);
+                if (op + sumd <= sm.bud_phase) { ok = 1; lbase = atomicAdd(&sm.lcnt[nx], ctot); }
+            }
+        }
+        ok = __shfl_sync(kFull, ok, 0);
+        lbase = __shfl_sync(kFull, lbase, 0);
+        if (ok) {
+#pragma unroll
+            for (int r = 0; r < 4; r++) {
+                if ((cm >> r) & 1u) {
+                    const int pos = lbase + coff[r] + __popc(cb[r] & lt);
+                    if (pos < kLCap) {
+                        sm.lv[nx][pos] = vv[r];
+                        sm.ld[nx][pos] = dd[r];
+                        sm.lb[nx][pos] = bb[r];
+                        lm |= 1u << r;
+                    }
+                }
+            }
+        }
+    }
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        const bool tog = ((wm >> r) & 1u) && dd[r] > 0 && !((lm >> r) & 1u);
+        const unsigned bg = __ballot_sync(kFull, tog);
+        if (bg) {
+            const int c = __popc(bg);
+            if (gcnt + c > kGStage) gq_flush(A, sm, wib, gcnt);
+            if (tog) {
+                const int pos = gcnt + __popc(bg & lt);
+                sm.gv[wib][pos] = vv[r];
+                sm.gd[wib][pos] = dd[r];
+                sm.gb[wib][pos] = bb[r];
+            }
+            gcnt += c;
+        }
+    }
+    __syncwarp();
+}
+
+__device__ __forceinline__ uint64_t deg_policy()
+{
+#if KC_DEG_EVICT_LAST
+    return l2_evict_last_policy();
+#else
+    return 0;
+#endif
+}
+
 __device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
 {
     const uint32_t bit = 1u << (v & 31);
-    return (atomicOr(A.claimed + (v >> 5), bit) & bit) == 0u;
+    return (atom_or_claim(A.claimed + (v >> 5), bit, deg_policy()) & bit) == 0u;
 }
 
 // --------------------------------------------------------- arc walking
@@ -487,11 +596,22 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int k, int nx
 #pragma unroll
     for (int r = 0; r < 4; r++)
         if (won[r]) A.core[uu[r]] = k;
+#if KC_ROUTE4
+    unsigned wm = 0;
 #pragma unroll
     for (int r = 0; r < 4; r++) {
-        if (won[r] && b1[r] > b0[r]) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[r]));
+        if (won[r] && b1[r] > b0[r]) prefetch_row(A.colidx, b0[r], b1[r]);
+        if (won[r]) wm |= 1u << r;
+    }
+    route_won4(A, sm, wib, wm, uu[0], uu[1], uu[2], uu[3], (int32_t)(b1[0] - b0[0]), (int32_t)(b1[1] - b0[1]),
+               (int32_t)(b1[2] - b0[2]), (int32_t)(b1[3] - b0[3]), b0[0], b0[1], b0[2], b0[3], nx, gcnt);
+#else
+#pragma unroll
+    for (int r = 0; r < 4; r++) {
+        if (won[r] && b1[r] > b0[r]) prefetch_row(A.colidx, b0[r], b1[r]);
         route_won(A, sm, wib, won[r], uu[r], (int32_t)(b1[r] - b0[r]), b0[r], nx, gcnt);
     }
+#endif
 }
 
 // Walk arcs [a0,a1) of a frontier whose entries are i = [s,e) with arc
@@ -506,6 +626,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
                                      bool use_bloom, bool atom_only, int &lmin, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
+    const uint64_t pol = deg_policy();
     // first entry: largest i in [s,e) with P(i) <= a0 (32-ary search)
     int64_t lo = s, hi = e;
     while (true) {
@@ -521,6 +642,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
     }
     int64_t i = lo;
     int64_t a = a0;
+    if (lane == 0) PROBE_W(10, threadIdx.x >> 5);
     while (a < a1) {
         const int64_t j = i + lane;
         int64_t wq = LLONG_MAX, wbeg = 0;
@@ -566,20 +688,24 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
                 for (int r = 0; r < kUnroll; r++)
                     if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
             }
+            if (lane == 0) PROBE_W(13, (threadIdx.x >> 5) | ((int64_t)u[0] << 16));
             int32_t d[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++)
-                d[r] = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_cg_i32(A.deg + u[r]));
+                d[r] = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
             int old[kUnroll];
 #pragma unroll
-            for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atomicSub(A.deg + u[r], 1) : INT_MIN;
+            for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
             unsigned hm = 0;
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
                 if (old[r] == k + 1) hm |= 1u << r;
                 else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
             }
-            if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, k, nx, u[0], u[1], u[2], u[3], hm, gcnt);
+            const unsigned hb = __ballot_sync(kFull, hm != 0);
+            if (lane == 0) PROBE_W(11, (threadIdx.x >> 5) | ((int64_t)__popc(hb) << 8) | ((int64_t)old[0] << 16));
+            if (hb) handle_hits(A, sm, k, nx, u[0], u[1], u[2], u[3], hm, gcnt);
+            if (lane == 0) PROBE_W(12, threadIdx.x >> 5);
             a = an;
         }
         a = limit;
@@ -600,13 +726,31 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         if (threadIdx.x == 0) PROBE(1, L);
         if (L == 0) break;
         // arc prefix of the list
-        const int64_t dv = threadIdx.x < L ? (int64_t)sm.ld[cur][threadIdx.x] : 0;
-        const unsigned long long ex = block_excl_scan(sm, (unsigned long long)dv);
-        if (threadIdx.x < L) sm.lpre[threadIdx.x] = (int64_t)ex;
-        const int64_t T = (int64_t)sm.tot_q;
         const int nx = cur ^ 1;
-        if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; sm.larc[nx] = 0; }
-        __syncthreads();
+        int64_t T;
+        if (KC_FASTSUB && L <= 32) {  // one warp: no block-wide scan
+            if (threadIdx.x < 32) {
+                const int lane = threadIdx.x;
+                const int64_t dv = lane < L ? (int64_t)sm.ld[cur][lane] : 0;
+                int64_t incl = dv;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int64_t t = __shfl_up_sync(kFull, incl, o);
+                    if (lane >= o) incl += t;
+                }
+                if (lane < L) sm.lpre[lane] = incl - dv;
+                if (lane == 31) { sm.lpre[L] = incl; sm.tot_q = (unsigned long long)incl; sm.lcnt[nx] = 0; sm.larc[nx] = 0; }
+            }
+            __syncthreads();
+            T = (int64_t)sm.tot_q;
+        } else {
+            const int64_t dv = threadIdx.x < L ? (int64_t)sm.ld[cur][threadIdx.x] : 0;
+            const unsigned long long ex = block_excl_scan(sm, (unsigned long long)dv);
+            if (threadIdx.x < L) sm.lpre[threadIdx.x] = (int64_t)ex;
+            T = (int64_t)sm.tot_q;
+            if (threadIdx.x == 0) { sm.lpre[L] = T; sm.lcnt[nx] = 0; sm.larc[nx] = 0; }
+            __syncthreads();
+        }
         if (threadIdx.x == 0) PROBE(2, T);
         int64_t C = (T + kWarps - 1) / kWarps;
         C = ((C + kBatch - 1) / kBatch) * kBatch;
@@ -615,9 +759,12 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         walked += T;
         if (subs) { *subs += 1; *tmax = max(*tmax, T); }
         if (threadIdx.x == 0) PROBE(3, sm.lcnt[nx]);
-        __syncthreads();
-        if (threadIdx.x == 0) PROBE(4, 0);
-        if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
+        if (!KC_FASTSUB) {
+            __syncthreads();
+            if (threadIdx.x == 0) { sm.lcnt[cur] = 0; sm.larc[cur] = 0; }
+        }
+        // (KC_FASTSUB: the loop-top barrier orders the walk before the next
+        // read of lcnt; list `cur` is reset when it next becomes `nx`)
         cur = nx;
     }
     return walked;
@@ -706,6 +853,7 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
 {
     const int k = c.k;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const uint64_t pol = deg_policy();
     constexpr int CH = 32 * kScanItems;
     for (int64_t off = lo + (int64_t)wib * CH; off < hi; off += (int64_t)kWarps * CH) {
         int32_t vv[kScanItems], dd[kScanItems];
@@ -716,7 +864,7 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
             if (idx < hi) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)idx;
         }
 #pragma unroll
-        for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_cg_i32(A.deg + vv[j]) : -1;
+        for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_deg(A.deg + vv[j], pol) : -1;
         unsigned wm = 0, km = 0;
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
@@ -761,9 +909,14 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
                 }
             }
 #pragma unroll
-            for (int j = 0; j < kScanItems; j++) {
-                if (du[j] > 0) asm volatile("prefetch.global.L2 [%0];" ::"l"(A.colidx + b0[j]));
-                route_won(A, sm, wib, (wm >> j) & 1u, vv[j], du[j], b0[j], 0, gcnt);
+            for (int j = 0; j < kScanItems; j++)
+                if (du[j] > 0) prefetch_row(A.colidx, b0[j], b0[j] + du[j]);
+            if constexpr (KC_ROUTE4 && kScanItems == 4) {
+                route_won4(A, sm, wib, wm, vv[0], vv[1], vv[2], vv[3], du[0], du[1], du[2], du[3], b0[0], b0[1],
+                           b0[2], b0[3], 0, gcnt);
+            } else {
+#pragma unroll
+                for (int j = 0; j < kScanItems; j++) route_won(A, sm, wib, (wm >> j) & 1u, vv[j], du[j], b0[j], 0, gcnt);
             }
         }
     }
@@ -1146,6 +1299,14 @@ __global__ void k_leader(KArgs A, int32_t *phase_out)
     advance(c, sn, p);
     S->pub = c;
     *phase_out = c.phase;
+}
+
+// Hand the persisting L2 window of a call back to normal eviction priority
+// (stream-ordered, after k_persistent), so later kernels get the whole L2.
+__global__ void k_l2_release(const char *base, int64_t lines)
+{
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < lines; i += (int64_t)gridDim.x * blockDim.x)
+        asm volatile("applypriority.global.L2::evict_normal [%0], 128;" ::"l"(base + i * 128) : "memory");
 }
 
 __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan, int32_t bloom,

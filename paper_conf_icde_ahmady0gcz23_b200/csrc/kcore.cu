@@ -11,9 +11,11 @@
 
 #include <cstdio>
 #include <cstring>
+#include <algorithm>
 #include <mutex>
 
 using namespace kc;
+
 
 namespace {
 
@@ -23,6 +25,7 @@ struct DevInfo {
     int sms = 0;
     int occ = 0;  // resident CTAs of k_persistent per SM
     int major = 0, minor = 0;
+    int persist_max = 0, window_max = 0;  // cudaDevAttrMaxPersistingL2CacheSize / AccessPolicyMaxWindowSize
     bool init = false;
 };
 
@@ -42,6 +45,8 @@ int dev_info(DevInfo &out)
         cudaDeviceGetAttribute(&d.major, cudaDevAttrComputeCapabilityMajor, dev);
         cudaDeviceGetAttribute(&d.minor, cudaDevAttrComputeCapabilityMinor, dev);
         if (d.major != 10) return KCORE_EUNSUPPORTED;
+        cudaDeviceGetAttribute(&d.persist_max, cudaDevAttrMaxPersistingL2CacheSize, dev);
+        cudaDeviceGetAttribute(&d.window_max, cudaDevAttrMaxAccessPolicyWindowSize, dev);
         const int smem = (int)sizeof(Smem);
         if (cudaFuncSetAttribute(k_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess ||
             cudaFuncSetAttribute(k_phase, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
@@ -83,7 +88,6 @@ size_t carve(void *base, int64_t n, Carve *c)
     const size_t nn = (size_t)(n > 0 ? n : 1);
     t.S = (State *)take(sizeof(State));
     t.order = (int32_t *)take(sizeof(int32_t) * nn);
-    t.claimed = (uint32_t *)take(sizeof(uint32_t) * ((nn + 31) / 32));
     t.gq_v = (int32_t *)take(sizeof(int32_t) * nn);
     t.gq_beg = (int64_t *)take(sizeof(int64_t) * nn);
     t.gq_arc = (int64_t *)take(sizeof(int64_t) * (nn + 1));
@@ -91,6 +95,8 @@ size_t carve(void *base, int64_t n, Carve *c)
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     t.seg1 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
+    // claim bits and working degrees adjacent: one L2 access-policy window
+    t.claimed = (uint32_t *)take(sizeof(uint32_t) * ((nn + 31) / 32));
     t.deg = (int32_t *)take(sizeof(int32_t) * nn);
     if (c) *c = t;
     return off;
@@ -196,6 +202,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     bool own_ws = false;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int32_t *d_phase = nullptr;
+    int64_t l2_lines = 0;
+    const char *l2_base = nullptr;
     State hS;
     Carve cv;
     KArgs A;
@@ -234,9 +242,46 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     KC_CUDA(cudaGetLastError());
     if (stats) KC_CUDA(cudaEventRecord(ev0, st));
     if (algo == KCORE_ALGO_PERSISTENT) {
-        void *args[] = {&A};
-        KC_CUDA(cudaLaunchCooperativeKernel((const void *)k_persistent, dim3(grid), dim3(kBlock), args,
-                                            smem, st));
+        const bool persist = !(opt && (opt->flags & KCORE_FLAG_NO_L2_PERSIST)) && di.persist_max > 0 &&
+                             di.window_max > 0;
+        if (persist) {
+            // persisting L2 window over the scattered working set (claim bits +
+            // working degrees): the adjacency stream of the heavy levels must not
+            // evict it.  The set-aside is raised to the
+            // window size (device limit, never lowered) and the lines are handed
+            // back to normal priority by k_l2_release after the kernel.
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(grid);
+            cfg.blockDim = dim3(kBlock);
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = st;
+            cudaLaunchAttribute at[2];
+            at[0].id = cudaLaunchAttributeCooperative;
+            at[0].val.cooperative = 1;
+            const size_t wbytes = std::min((size_t)((char *)(cv.deg + n) - (char *)cv.claimed), (size_t)di.window_max);
+            size_t lim = 0;
+            cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize);
+            const size_t want = std::min(wbytes, (size_t)di.persist_max);
+            if (lim < want) {
+                KC_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
+                KC_CUDA(cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize));
+            }
+            at[1].id = cudaLaunchAttributeAccessPolicyWindow;
+            at[1].val.accessPolicyWindow.base_ptr = cv.claimed;
+            at[1].val.accessPolicyWindow.num_bytes = wbytes;
+            at[1].val.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)lim / (double)wbytes);
+            at[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+            at[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+            cfg.attrs = at;
+            cfg.numAttrs = 2;
+            KC_CUDA(cudaLaunchKernelEx(&cfg, k_persistent, A));
+            l2_lines = (int64_t)(wbytes / 128);
+            l2_base = (const char *)cv.claimed;
+        } else {
+            void *args[] = {&A};
+            KC_CUDA(cudaLaunchCooperativeKernel((const void *)k_persistent, dim3(grid), dim3(kBlock), args,
+                                                smem, st));
+        }
     } else {
         KC_CUDA(cudaMallocAsync((void **)&d_phase, sizeof(int32_t), st));
         int32_t ph = PH_INIT;
@@ -251,6 +296,10 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         }
     }
     if (stats) KC_CUDA(cudaEventRecord(ev1, st));
+    if (l2_lines > 0) {
+        k_l2_release<<<std::min<int64_t>((l2_lines + 255) / 256, 4 * di.sms), 256, 0, st>>>(l2_base, l2_lines);
+        KC_CUDA(cudaGetLastError());
+    }
     if (opt && opt->order_out)
         KC_CUDA(cudaMemcpyAsync(opt->order_out, cv.order, sizeof(int32_t) * (size_t)n,
                                 cudaMemcpyDeviceToDevice, st));
