@@ -160,6 +160,49 @@ const char *kcore_strerror(int status);
 const char *kcore_version(void);
 
 /* ---------------------------------------------------------------------------
+ * Outputs derived from a decomposition.  `core` is a
+ * DEVICE int32[n] core array (e.g. kcore_decompose's core_out).  All three
+ * synchronise `stream` (they return host counts).  Vertex lists are in
+ * increasing vertex id.
+ * ------------------------------------------------------------------------- */
+
+/* The k-shell {v : core(v) == k} (Sec. II-A).  vertices_out: DEVICE
+ * int32 with room for the shell (NULL: count only).  *count_out (HOST) = its
+ * size. */
+int kcore_kshell(const int32_t *core, int64_t n, int32_t k, int32_t *vertices_out, int64_t *count_out,
+                 void *stream);
+
+/* Membership mask of the k-core {v : core(v) >= k} (the k-cores are
+ * nested).  mask_out: DEVICE uint8[n] (1 = in the k-core).  *count_out
+ * (HOST, may be NULL) = k-core size. */
+int kcore_kcore_mask(const int32_t *core, int64_t n, int32_t k, uint8_t *mask_out, int64_t *count_out,
+                     void *stream);
+
+/* The k-core as an induced subgraph (k-core as the pre-processing of
+ * dense-subgraph mining), vertices renumbered in increasing original id.
+ * Two calls: with sub_rowptr == NULL only *nk_out / *mk_out (HOST) are
+ * computed; then with DEVICE buffers sub_rowptr int64[nk+1], sub_colidx
+ * int32[mk], vmap_out int32[nk] (vmap_out[new] = original id), which are
+ * filled (rows sorted, symmetric, like the input). */
+int kcore_kcore_subgraph(const int64_t *rowptr, const int32_t *colidx, const int32_t *core, int64_t n,
+                         int64_t m, int32_t k, int64_t *nk_out, int64_t *mk_out, int64_t *sub_rowptr,
+                         int32_t *sub_colidx, int32_t *vmap_out, void *stream);
+
+/* ---------------------------------------------------------------------------
+ * MPM: the paper's h-index algorithm family (P:L27,
+ * P:L65-69, Fig. 2) in the bulk-synchronous form of Medusa-MPM:
+ *   a_0(v) = deg(v);  a_t(v) = max{h : |{u in N(v) : a_{t-1}(u) >= h}| >= h}
+ * until an iteration changes nothing (then a = core) or `max_iters`
+ * iterations have run (max_iters < 0: no limit).  DEVICE rowptr/colidx/a_out
+ * (int32[n], the last iterate).  *iters_out (HOST, may be NULL) = iterations
+ * that changed at least one value.  One persistent cooperative kernel;
+ * scratch (about 24 n bytes) is allocated stream-ordered.  Synchronises
+ * `stream`.  stats (may be NULL): levels = phases = iterations, scanned =
+ * sum of active-set sizes, arcs_walked = arcs gathered, kernel_ms. */
+int kcore_mpm(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m, int32_t *a_out,
+              int64_t max_iters, int64_t *iters_out, void *stream, kcore_stats *stats);
+
+/* ---------------------------------------------------------------------------
  * Multi-GPU: 1D vertex-range ownership (north star; the paper's multi-GPU
  * future work, with owner routing instead of a master GPU).
  * Rank r owns vertices [v_begin, v_end) and stores their rows:

@@ -13,6 +13,9 @@ file's header for the paper passages each function follows:
 * :func:`core_smallest_last`  -- smallest-last min-degree removal (ref [58]).
 * :func:`core_subsets`        -- literal subset definition, n <= 20.
 * :func:`hindex`              -- MPM h-index operator (Fig. 2).
+* :func:`kcore_members`       -- the k-core by its definition (repeated deletion).
+* :func:`induced_csr`         -- induced subgraph G[S], renumbered by increasing id.
+* :func:`mpm`                 -- synchronous MPM h-index iteration.
 * :func:`check_invariants`, :func:`check_certificate`, :func:`validate_csr`.
 """
 from __future__ import annotations
@@ -56,6 +59,10 @@ def _load():
         lib.oracle_check_invariants.argtypes = [ctypes.c_int64, I64P, I32P, I32P]
         lib.oracle_check_certificate.argtypes = [ctypes.c_int64, I64P, I32P, I32P, I32P]
         lib.oracle_validate_csr.argtypes = [ctypes.c_int64, ctypes.c_int64, I64P, I32P]
+        U8P = ctypes.POINTER(ctypes.c_uint8)
+        lib.oracle_kcore_members.argtypes = [ctypes.c_int64, I64P, I32P, ctypes.c_int64, U8P]
+        lib.oracle_induced_csr.argtypes = [ctypes.c_int64, I64P, I32P, U8P, I64P, I64P, I64P, I32P, I32P]
+        lib.oracle_mpm.argtypes = [ctypes.c_int64, I64P, I32P, ctypes.c_int64, I32P, I64P]
         _lib = lib
     return _lib
 
@@ -148,3 +155,41 @@ def validate_csr(rowptr, colidx) -> int:
     rp, ci, n = _csr(rowptr, colidx)
     return int(_load().oracle_validate_csr(n, ci.shape[0], _p64(rp), _p32(ci)))
 
+
+
+def _u8p(a):
+    return a.ctypes.data_as(ctypes.POINTER(ctypes.c_uint8))
+
+
+def kcore_members(rowptr, colidx, k: int):
+    """uint8 mask of the k-core, by repeated deletion of degree < k."""
+    rp, ci, n = _csr(rowptr, colidx)
+    mask = np.empty(max(n, 1), dtype=np.uint8)
+    if _load().oracle_kcore_members(n, _p64(rp), _p32(ci), int(k), _u8p(mask)) != 0:
+        raise RuntimeError("oracle_kcore_members failed")
+    return mask[:n]
+
+
+def induced_csr(rowptr, colidx, keep):
+    """(rowptr, colidx, vmap) of G[{v: keep[v]}], renumbered by increasing id."""
+    rp, ci, n = _csr(rowptr, colidx)
+    kp = np.ascontiguousarray(np.asarray(keep), dtype=np.uint8)
+    nk, mk = ctypes.c_int64(0), ctypes.c_int64(0)
+    lib = _load()
+    lib.oracle_induced_csr(n, _p64(rp), _p32(ci), _u8p(kp), ctypes.byref(nk), ctypes.byref(mk), None, None, None)
+    orp = np.zeros(nk.value + 1, dtype=np.int64)
+    oci = np.empty(max(mk.value, 1), dtype=np.int32)
+    vm = np.empty(max(nk.value, 1), dtype=np.int32)
+    lib.oracle_induced_csr(n, _p64(rp), _p32(ci), _u8p(kp), ctypes.byref(nk), ctypes.byref(mk), _p64(orp),
+                           _p32(oci), _p32(vm))
+    return orp, oci[:mk.value], vm[:nk.value]
+
+
+def mpm(rowptr, colidx, max_iters: int = -1):
+    """Synchronous MPM: (a, iterations).  a = core at convergence."""
+    rp, ci, n = _csr(rowptr, colidx)
+    a = np.empty(max(n, 1), dtype=np.int32)
+    it = ctypes.c_int64(0)
+    if _load().oracle_mpm(n, _p64(rp), _p32(ci), int(max_iters), _p32(a), ctypes.byref(it)) != 0:
+        raise RuntimeError("oracle_mpm failed")
+    return a[:n], int(it.value)

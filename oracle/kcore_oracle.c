@@ -393,3 +393,113 @@ int oracle_validate_csr(int64_t n, int64_t arcs, const int64_t *rowptr, const in
             if (!has_arc(rowptr, colidx, colidx[e], (int32_t)v)) return 5;
     return 0;
 }
+
+/* ------------------------------------------------------------------------ */
+/* (8) The k-core itself ("the largest induced subgraph with minimum  */
+/*     degree k"), by its definition: start from S = V and delete vertices   */
+/*     with fewer than k neighbours in S until none is left (a queue makes   */
+/*     each deletion O(deg)).  in_core[v] = 1 iff v is in the k-core.        */
+/*     Uses no core numbers.                                                  */
+/* ------------------------------------------------------------------------ */
+int oracle_kcore_members(int64_t n, const int64_t *rowptr, const int32_t *colidx, int64_t k,
+                         uint8_t *in_core)
+{
+    if (n < 0) return OR_EINVAL;
+    if (n == 0) return OR_OK;
+    int64_t *d = (int64_t *)malloc(sizeof(int64_t) * (size_t)n);
+    int32_t *q = (int32_t *)malloc(sizeof(int32_t) * (size_t)n);
+    if (!d || !q) { free(d); free(q); return OR_ENOMEM; }
+    int64_t qh = 0, qt = 0;
+    for (int64_t v = 0; v < n; v++) {
+        in_core[v] = 1;
+        d[v] = rowptr[v + 1] - rowptr[v];
+        if (d[v] < k) { in_core[v] = 0; q[qt++] = (int32_t)v; }
+    }
+    while (qh < qt) {
+        int32_t v = q[qh++];
+        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; e++) {
+            int32_t u = colidx[e];
+            if (!in_core[u]) continue;
+            if (--d[u] < k) { in_core[u] = 0; q[qt++] = u; }
+        }
+    }
+    free(d); free(q);
+    return OR_OK;
+}
+
+/* ------------------------------------------------------------------------ */
+/* (9) Induced subgraph G[S] for S = {v : keep[v]}, vertices renumbered in   */
+/*     increasing original id (vmap[new] = old), rows sorted.  Call with     */
+/*     rp_out == NULL to get the sizes only.                                  */
+/* ------------------------------------------------------------------------ */
+int oracle_induced_csr(int64_t n, const int64_t *rowptr, const int32_t *colidx, const uint8_t *keep,
+                       int64_t *nk, int64_t *mk, int64_t *rp_out, int32_t *ci_out, int32_t *vmap_out)
+{
+    if (n < 0) return OR_EINVAL;
+    int32_t *newid = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n > 0 ? n : 1));
+    if (!newid) return OR_ENOMEM;
+    int64_t cnt = 0, arcs = 0;
+    for (int64_t v = 0; v < n; v++) newid[v] = keep[v] ? (int32_t)cnt++ : -1;
+    if (rp_out) rp_out[0] = 0;
+    for (int64_t v = 0; v < n; v++) {
+        if (!keep[v]) continue;
+        if (vmap_out) vmap_out[newid[v]] = (int32_t)v;
+        for (int64_t e = rowptr[v]; e < rowptr[v + 1]; e++) {
+            int32_t u = colidx[e];
+            if (!keep[u]) continue;
+            if (ci_out) ci_out[arcs] = newid[u];
+            arcs++;
+        }
+        if (rp_out) rp_out[newid[v] + 1] = arcs;
+    }
+    *nk = cnt;
+    *mk = arcs;
+    free(newid);
+    return OR_OK;
+}
+
+/* ------------------------------------------------------------------------ */
+/* (10) MPM [63] as the paper describes it (Fig. 2) in the        */
+/*      bulk-synchronous form of Medusa-MPM (every vertex reads its  */
+/*      neighbours' estimates of the previous iteration; a global flag says  */
+/*      whether another iteration is needed):                                 */
+/*        a_0(v) = deg(v);                                                    */
+/*        a_{t+1}(v) = h-index of the multiset {a_t(u) : (u,v) in E}          */
+/*      using oracle_hindex (sort non-increasing, max i with A[i] >= i).      */
+/*      Runs until an iteration changes nothing or `max_iters` iterations    */
+/*      have run (max_iters < 0: no limit).  a_out = the last iterate;       */
+/*      *iters_out = number of iterations that changed at least one value.   */
+/*      At convergence a = core.                                      */
+/* ------------------------------------------------------------------------ */
+int oracle_mpm(int64_t n, const int64_t *rowptr, const int32_t *colidx, int64_t max_iters,
+               int32_t *a_out, int64_t *iters_out)
+{
+    if (n < 0) return OR_EINVAL;
+    *iters_out = 0;
+    if (n == 0) return OR_OK;
+    int64_t md = 0;
+    for (int64_t v = 0; v < n; v++)
+        if (rowptr[v + 1] - rowptr[v] > md) md = rowptr[v + 1] - rowptr[v];
+    int32_t *prev = (int32_t *)malloc(sizeof(int32_t) * (size_t)n);
+    int32_t *vals = (int32_t *)malloc(sizeof(int32_t) * (size_t)(md > 0 ? md : 1));
+    if (!prev || !vals) { free(prev); free(vals); return OR_ENOMEM; }
+    for (int64_t v = 0; v < n; v++) a_out[v] = (int32_t)(rowptr[v + 1] - rowptr[v]);
+    int64_t it = 0;
+    while (max_iters < 0 || it < max_iters) {
+        memcpy(prev, a_out, sizeof(int32_t) * (size_t)n);
+        int changed = 0;
+        for (int64_t v = 0; v < n; v++) {
+            int64_t c = 0;
+            for (int64_t e = rowptr[v]; e < rowptr[v + 1]; e++) vals[c++] = prev[colidx[e]];
+            int32_t h = oracle_hindex(vals, c);
+            if (h < 0) { free(prev); free(vals); return OR_ENOMEM; }
+            if (h != prev[v]) changed = 1;
+            a_out[v] = h;
+        }
+        if (!changed) break;
+        it++;
+    }
+    *iters_out = it;
+    free(prev); free(vals);
+    return OR_OK;
+}

@@ -13,6 +13,9 @@ Entry points mirror the C names:
 * :func:`kcore_decompose_mg`    -- multi-GPU, 1-D vertex-range ownership (NCCL).
 * :func:`kcore_decompose_mg_virtual` -- the multi-GPU protocol with virtual
   ranks on one GPU (testing).
+* :func:`kcore_kshell`, :func:`kcore_kcore_mask`, :func:`kcore_kcore_subgraph` -- k-shell /
+  k-core outputs of a decomposition.
+* :func:`kcore_mpm`             -- the MPM h-index iteration (the paper's second family).
 * :func:`kcore_validate_csr`, :func:`kcore_workspace_size`, :func:`kcore_strerror`.
 """
 from __future__ import annotations
@@ -42,7 +45,7 @@ EXPORTS = (
     "kcore_decompose", "kcore_decompose_ex", "kcore_decompose_host", "kcore_workspace_size",
     "kcore_validate_csr", "kcore_strerror", "kcore_version", "kcore_decompose_mg",
     "kcore_decompose_mg_virtual", "kcore_nccl_unique_id", "kcore_nccl_comm_init",
-    "kcore_nccl_comm_destroy",
+    "kcore_nccl_comm_destroy", "kcore_kshell", "kcore_kcore_mask", "kcore_kcore_subgraph", "kcore_mpm",
 )
 
 
@@ -126,6 +129,11 @@ def _load():
         lib.kcore_nccl_unique_id.argtypes = [vp]
         lib.kcore_nccl_comm_init.argtypes = [ctypes.POINTER(vp), i32, vp, i32]
         lib.kcore_nccl_comm_destroy.argtypes = [vp]
+        i64p = ctypes.POINTER(ctypes.c_int64)
+        lib.kcore_kshell.argtypes = [vp, i64, i32, vp, i64p, vp]
+        lib.kcore_kcore_mask.argtypes = [vp, i64, i32, vp, i64p, vp]
+        lib.kcore_kcore_subgraph.argtypes = [vp, vp, vp, i64, i64, i32, i64p, i64p, vp, vp, vp, vp]
+        lib.kcore_mpm.argtypes = [vp, vp, i64, i64, vp, i64, i64p, vp, ctypes.POINTER(_Stats)]
         _lib = lib
     return _lib
 
@@ -256,6 +264,97 @@ def kcore_decompose_mg_virtual(rowptr, colidx, nranks: int, *, stats: bool = Fal
     return (core, Stats._from(st)) if stats else core
 
 
+def _check_core(core):
+    import torch
+    if not core.is_cuda or core.dtype != torch.int32 or not core.is_contiguous():
+        raise TypeError("core must be a contiguous int32 CUDA tensor")
+
+
+def kcore_kshell(core, k: int):
+    """The k-shell {v : core[v] == k} as an int32 CUDA tensor of vertex ids (increasing)."""
+    import torch
+    _check_core(core)
+    n = core.numel()
+    cnt = ctypes.c_int64(0)
+    lib = _load()
+    with torch.cuda.device(core.device):
+        rc = lib.kcore_kshell(core.data_ptr() if n else None, n, int(k), None, ctypes.byref(cnt),
+                              _stream_ptr(core.device))
+        if rc != KCORE_OK:
+            raise KcoreError(rc, "kcore_kshell")
+        out = torch.empty(cnt.value, dtype=torch.int32, device=core.device)
+        if cnt.value:
+            rc = lib.kcore_kshell(core.data_ptr(), n, int(k), out.data_ptr(), ctypes.byref(cnt),
+                                  _stream_ptr(core.device))
+            if rc != KCORE_OK:
+                raise KcoreError(rc, "kcore_kshell")
+    return out
+
+
+def kcore_kcore_mask(core, k: int):
+    """(uint8 CUDA mask of the k-core {v : core[v] >= k}, its size)."""
+    import torch
+    _check_core(core)
+    n = core.numel()
+    mask = torch.empty(n, dtype=torch.uint8, device=core.device)
+    cnt = ctypes.c_int64(0)
+    with torch.cuda.device(core.device):
+        rc = _load().kcore_kcore_mask(core.data_ptr() if n else None, n, int(k), mask.data_ptr() if n else None,
+                                      ctypes.byref(cnt), _stream_ptr(core.device))
+    if rc != KCORE_OK:
+        raise KcoreError(rc, "kcore_kcore_mask")
+    return mask, int(cnt.value)
+
+
+def kcore_kcore_subgraph(rowptr, colidx, core, k: int):
+    """The induced k-core subgraph: (sub_rowptr int64, sub_colidx int32, vmap int32) CUDA
+    tensors, vertices renumbered in increasing original id (vmap[new] = old)."""
+    import torch
+    _check_csr_tensors(rowptr, colidx)
+    _check_core(core)
+    n = rowptr.numel() - 1
+    m = colidx.numel()
+    nk, mk = ctypes.c_int64(0), ctypes.c_int64(0)
+    lib = _load()
+    dev = rowptr.device
+    cp = colidx.data_ptr() if m else None
+    with torch.cuda.device(dev):
+        rc = lib.kcore_kcore_subgraph(rowptr.data_ptr(), cp, core.data_ptr() if n else None, n, m, int(k),
+                                      ctypes.byref(nk), ctypes.byref(mk), None, None, None, _stream_ptr(dev))
+        if rc != KCORE_OK:
+            raise KcoreError(rc, "kcore_kcore_subgraph")
+        srp = torch.empty(nk.value + 1, dtype=torch.int64, device=dev)
+        sci = torch.empty(max(mk.value, 1), dtype=torch.int32, device=dev)
+        vm = torch.empty(max(nk.value, 1), dtype=torch.int32, device=dev)
+        rc = lib.kcore_kcore_subgraph(rowptr.data_ptr(), cp, core.data_ptr() if n else None, n, m, int(k),
+                                      ctypes.byref(nk), ctypes.byref(mk), srp.data_ptr(), sci.data_ptr(),
+                                      vm.data_ptr(), _stream_ptr(dev))
+    if rc != KCORE_OK:
+        raise KcoreError(rc, "kcore_kcore_subgraph")
+    return srp, sci[:mk.value], vm[:nk.value]
+
+
+def kcore_mpm(rowptr, colidx, *, max_iters: int = -1, a_out=None, stats: bool = False):
+    """MPM h-index iteration (bulk-synchronous as P:L388): (a, iterations[, Stats]).
+    a = core at convergence; with max_iters >= 0, the iterate after that many iterations."""
+    import torch
+    _check_csr_tensors(rowptr, colidx)
+    dev = rowptr.device
+    n = rowptr.numel() - 1
+    m = colidx.numel()
+    if a_out is None:
+        a_out = torch.empty(max(n, 0), dtype=torch.int32, device=dev)
+    it = ctypes.c_int64(0)
+    st = _Stats()
+    with torch.cuda.device(dev):
+        rc = _load().kcore_mpm(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
+                               a_out.data_ptr() if n else None, int(max_iters), ctypes.byref(it),
+                               _stream_ptr(dev), ctypes.byref(st) if stats else None)
+    if rc != KCORE_OK:
+        raise KcoreError(rc, "kcore_mpm")
+    return (a_out, int(it.value), Stats._from(st)) if stats else (a_out, int(it.value))
+
+
 from .parallel import (  # noqa: E402
     NcclComm, kcore_decompose_mg, owner_ranges, local_csr, gather_cores,
 )
@@ -264,4 +363,5 @@ __all__ = [
     "kcore_decompose", "kcore_decompose_host", "kcore_decompose_mg", "kcore_decompose_mg_virtual",
     "kcore_validate_csr", "kcore_workspace_size", "strerror", "version", "Stats", "KcoreError",
     "NcclComm", "owner_ranges", "local_csr", "gather_cores", "EXPORTS", "LIB_PATH",
+    "kcore_kshell", "kcore_kcore_mask", "kcore_kcore_subgraph", "kcore_mpm",
 ]

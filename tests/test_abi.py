@@ -66,6 +66,29 @@ def test_argument_errors_before_any_launch():
         kc.KCORE_EINVAL, kc.KCORE_EUNSUPPORTED)
 
 
+def test_output_and_mpm_argument_errors_before_any_launch():
+    lib = kc.library()
+    d = ctypes.c_void_p(0x1000)
+    cnt, cnt2 = ctypes.c_int64(7), ctypes.c_int64(7)
+    assert lib.kcore_kshell(d, -1, 0, d, ctypes.byref(cnt), None) == kc.KCORE_EINVAL
+    assert lib.kcore_kshell(None, 5, 0, d, ctypes.byref(cnt), None) == kc.KCORE_EINVAL
+    assert lib.kcore_kshell(None, 0, 3, None, ctypes.byref(cnt), None) == kc.KCORE_OK and cnt.value == 0
+    assert lib.kcore_kcore_mask(d, 5, 1, None, None, None) == kc.KCORE_EINVAL
+    assert lib.kcore_kcore_mask(d, 1 << 31, 1, d, None, None) == kc.KCORE_EINVAL
+    assert lib.kcore_kcore_subgraph(d, d, d, 4, 6, 1, None, ctypes.byref(cnt2), None, None, None,
+                                    None) == kc.KCORE_EINVAL
+    assert lib.kcore_kcore_subgraph(d, d, d, 4, 6, 1, ctypes.byref(cnt), ctypes.byref(cnt2), d, d, None,
+                                    None) == kc.KCORE_EINVAL  # filling needs vmap_out
+    assert lib.kcore_kcore_subgraph(None, None, None, 0, 0, 1, ctypes.byref(cnt), ctypes.byref(cnt2), None,
+                                    None, None, None) == kc.KCORE_OK
+    assert cnt.value == 0 and cnt2.value == 0
+    it = ctypes.c_int64(5)
+    assert lib.kcore_mpm(d, d, -1, 0, d, -1, ctypes.byref(it), None, None) == kc.KCORE_EINVAL
+    assert lib.kcore_mpm(d, None, 4, 6, d, -1, ctypes.byref(it), None, None) == kc.KCORE_EINVAL
+    assert lib.kcore_mpm(None, None, 0, 0, None, -1, ctypes.byref(it), None, None) == kc.KCORE_OK
+    assert it.value == 0
+
+
 def test_no_cpu_fallback_in_product_package():
     """The product package never imports the oracle or any CPU decomposition."""
     pkg = os.path.join(ROOT, "paper_conf_icde_ahmady0gcz23_b200")
