@@ -16,6 +16,12 @@
 
 using namespace kc;
 
+// L2 property of the window's lines beyond hitRatio (the set-aside is smaller
+// than the window on some parts)
+#ifndef KC_MISS_PROP
+#define KC_MISS_PROP cudaAccessPropertyNormal
+#endif
+
 
 namespace {
 
@@ -266,12 +272,20 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
                 KC_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
                 KC_CUDA(cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize));
             }
+            if (lim * 4 < wbytes) {
+                // no usable set-aside (e.g. a profiler pinned the limit at 0): a window
+                // with hitRatio ~ 0 would mark deg streaming -- launch without one
+                void *args[] = {&A};
+                KC_CUDA(cudaLaunchCooperativeKernel((const void *)k_persistent, dim3(grid), dim3(kBlock), args,
+                                                    smem, st));
+                goto launched;
+            }
             at[1].id = cudaLaunchAttributeAccessPolicyWindow;
             at[1].val.accessPolicyWindow.base_ptr = cv.claimed;
             at[1].val.accessPolicyWindow.num_bytes = wbytes;
             at[1].val.accessPolicyWindow.hitRatio = (float)std::min(1.0, (double)lim / (double)wbytes);
             at[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-            at[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+            at[1].val.accessPolicyWindow.missProp = KC_MISS_PROP;
             cfg.attrs = at;
             cfg.numAttrs = 2;
             KC_CUDA(cudaLaunchKernelEx(&cfg, k_persistent, A));
@@ -295,6 +309,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
             if (++guard > (1 << 28)) { rc = KCORE_ECUDA; goto done; }
         }
     }
+launched:
     if (stats) KC_CUDA(cudaEventRecord(ev1, st));
     if (l2_lines > 0) {
         k_l2_release<<<std::min<int64_t>((l2_lines + 255) / 256, 4 * di.sms), 256, 0, st>>>(l2_base, l2_lines);
