@@ -1,4 +1,4 @@
-"""Summarise an ncu report of k_persistent into profiles/ (JSON + text).
+"""Summarise a one-kernel ncu report into profiles/ (JSON).
    python tools/ncu_summary.py gpurun_out/prof.ncu-rep profiles/ncu_r1_C4 [launches.csv]"""
 import csv, io, json, subprocess, sys
 
@@ -7,6 +7,7 @@ raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_outpu
 rows = list(csv.reader(io.StringIO(raw)))
 h, units, vals = rows[0], rows[1], rows[2]
 d = {h[i]: (vals[i], units[i]) for i in range(len(h))}
+KNAME = d.get("Kernel Name", ("?", ""))[0]
 
 
 def num(k):
@@ -41,7 +42,7 @@ stalls = {k.replace("smsp__pcsamp_warps_issue_stalled_", ""): num(k) for k in d
           if k.startswith("smsp__pcsamp_warps_issue_stalled_") and not k.endswith("not_issued")}
 tot = sum(v for v in stalls.values() if v) or 1
 stalls = {k: round(100 * v / tot, 1) for k, v in sorted(stalls.items(), key=lambda x: -(x[1] or 0)) if v}
-res = {"report": rep, "kernel": "kc::k_persistent", "duration_s": dur, "dram_bytes_read": rd, "dram_bytes_write": wr,
+res = {"report": rep, "kernel": KNAME, "duration_s": dur, "dram_bytes_read": rd, "dram_bytes_write": wr,
        "dram_bytes_per_launch": (rd or 0) + (wr or 0),
        "dram_GBps": ((rd or 0) + (wr or 0)) / dur / 1e9 if dur else None,
        "stall_pct": dict(list(stalls.items())[:12]), "metrics": summary}
