@@ -14,9 +14,10 @@
  * P:L187-298), re-designed for sm_100a as ONE persistent cooperative kernel
  * per call: deg init (Alg. 1 l.1), level scan (Alg. 2) fused with the
  * min-degree reduction for level skipping, peel sub-rounds (Alg. 3 l.12-24:
- * atomicSub returning the old value, append on old == k+1, restore on
- * old <= k, P:L322-334 / Fig. 6), with no host round-trip between levels or
- * sub-rounds.  See DESIGN.md.
+ * atomicSub returning the old value, append on old == k+1), with
+ * no host round-trip between levels or sub-rounds.  The degrees are a private
+ * working array, so the restore of Fig. 6 is not needed: core(v)
+ * is written once, when v is claimed (reading R10).
  *
  * Conventions shared by every entry point
  *  - n      : |V|, 0 <= n < 2^31 (vertex ids are int32).

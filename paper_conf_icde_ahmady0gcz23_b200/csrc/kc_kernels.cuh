@@ -11,12 +11,14 @@
 //                             alive-list compaction;
 //             then drains its local frontier breadth-first with CTA-local
 //             sub-rounds (__syncthreads only) -- the paper's block-local BFS
-//             of Alg. 3.  For every arc (v,u) (Alg. 3 l.19-24):
-//               if deg[u] > k: old = atomicSub(&deg[u],1)
-//                  old == k+1 -> u reached k: claim it, append it to the next
-//                                local frontier
-//                  old <= k   -> atomicAdd(&deg[u],1)  (restore, Fig. 6)
-//                  else       -> min_next = min(min_next, old-1)    (level skip)
+//             of Alg. 3.  For every arc (v,u) (Alg. 3 l.19-24)
+//             whose target passes the alive filter:
+//               old = atomicSub(&deg[u],1)
+//                  old == k+1 -> u reached k: claim it, core[u] = k, append it
+//                                to the next local frontier
+//                  old >  k+1 -> min_next = min(min_next, old-1)    (level skip)
+//             deg is a private working array (reading R10): removed
+//             targets take garbage decrements, so no restore (Fig. 6) is needed.
 //   HUB       vertices too big for one CTA (> kHub arcs) or overflowing a
 //             local frontier go to a global queue; a HUB phase splits that
 //             queue's ARCS evenly over every warp of the grid, then drains
