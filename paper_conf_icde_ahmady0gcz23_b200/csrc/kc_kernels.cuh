@@ -92,6 +92,15 @@ constexpr int kTraceFields = 8;
 #ifndef KC_ROUTE4
 #define KC_ROUTE4 1
 #endif
+#ifndef KC_CF_HUB
+#define KC_CF_HUB 0
+#endif
+#ifndef KC_CF_LOCAL
+#define KC_CF_LOCAL 0
+#endif
+#ifndef KC_CF_LOCAL_MIN
+#define KC_CF_LOCAL_MIN 0
+#endif
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
 #endif
@@ -595,6 +604,15 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int k, int nx
     bool won[4];
 #pragma unroll
     for (int r = 0; r < 4; r++) won[r] = ((hm >> r) & 1u) && claim(A, uu[r]);
+#ifdef KC_PROBE_W
+    {
+        int64_t dep = 0;
+#pragma unroll
+        for (int r = 0; r < 4; r++) dep += b0[r] + b1[r] + (won[r] ? 1 : 0);
+        dep = __reduce_add_sync(kFull, (unsigned)(dep & 0xffff));
+        if ((threadIdx.x & 31) == 0) PROBE_W(14, (threadIdx.x >> 5) | ((dep & 0xff) << 8));
+    }
+#endif
 #pragma unroll
     for (int r = 0; r < 4; r++)
         if (won[r]) A.core[uu[r]] = k;
@@ -625,7 +643,7 @@ __device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int k, int nx
 template <bool LOCAL>
 __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, const int cur, const int nx,
                                      int64_t s, int64_t e, int64_t ae, int64_t a0, int64_t a1,
-                                     bool use_bloom, bool atom_only, int &lmin, int &gcnt)
+                                     bool use_bloom, bool atom_only, int &lmin, int &gcnt, bool claim_filter = false)
 {
     const int lane = threadIdx.x & 31;
     const uint64_t pol = deg_policy();
@@ -689,6 +707,17 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
 #pragma unroll
                 for (int r = 0; r < kUnroll; r++)
                     if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
+            }
+            if (claim_filter) {
+                // exact dead-target filter: the claim bitmap (2 MB at C4, L1/L2
+                // resident) -- a set bit is final, a stale clear bit only costs
+                // the atomic we would have issued anyway
+                uint32_t cw[kUnroll];
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++) cw[r] = u[r] >= 0 ? A.claimed[u[r] >> 5] : 0u;
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++)
+                    if (u[r] >= 0 && ((cw[r] >> (u[r] & 31)) & 1u)) u[r] = -1;
             }
             if (lane == 0) PROBE_W(13, (threadIdx.x >> 5) | ((int64_t)u[0] << 16));
             int32_t d[kUnroll];
@@ -757,7 +786,9 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
         int64_t C = (T + kWarps - 1) / kWarps;
         C = ((C + kBatch - 1) / kBatch) * kBatch;
         const int64_t a0 = (int64_t)wib * C;
-        if (a0 < T) walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, atom_only, lmin, gcnt);
+        if (a0 < T)
+            walk<true>(A, sm, k, cur, nx, 0, L, T, a0, min(a0 + C, T), use_bloom, atom_only, lmin, gcnt,
+                       KC_CF_LOCAL && T >= KC_CF_LOCAL_MIN);
         walked += T;
         if (subs) { *subs += 1; *tmax = max(*tmax, T); }
         if (threadIdx.x == 0) PROBE(3, sm.lcnt[nx]);
@@ -1025,7 +1056,7 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_HUB;
     const int64_t a0 = c.as + gw * C;
     if (a0 < c.ae)
-        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt);
+        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt, KC_CF_HUB);
     int64_t walked = cta_arcs;
     __syncthreads();
     cta_time(A, c, 1);
@@ -1225,7 +1256,7 @@ __device__ __forceinline__ void init_ctrl(Ctrl &z)
     z.light = 0;
 }
 
-__global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
+__global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant__ KArgs A)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -1275,7 +1306,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(KArgs A)
 // -------------------------------------------- host-driven ablation kernels
 // (KCORE_ALGO_HOSTLOOP: the paper's Alg. 1 structure -- one launch per phase
 // and a host read-back of the phase after each.  No solo phases.)
-__global__ void __launch_bounds__(kBlock, 1) k_phase(KArgs A)
+__global__ void __launch_bounds__(kBlock, 1) k_phase(const __grid_constant__ KArgs A)
 {
     extern __shared__ __align__(16) unsigned char smem_raw[];
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
@@ -1290,7 +1321,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(KArgs A)
     else run_phase(A, c, sm, blockIdx.x, gridDim.x);
 }
 
-__global__ void k_leader(KArgs A, int32_t *phase_out)
+__global__ void k_leader(const __grid_constant__ KArgs A, int32_t *phase_out)
 {
     State *S = A.S;
     const Params p = S->prm;

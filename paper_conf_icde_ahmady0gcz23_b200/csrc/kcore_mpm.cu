@@ -235,7 +235,7 @@ __device__ void big_vertex(const MArgs &A, MSmem &sm, int32_t v, int t)
     }
 }
 
-__global__ void __launch_bounds__(kB, 1) k_mpm(MArgs A)
+__global__ void __launch_bounds__(kB, 1) k_mpm(const __grid_constant__ MArgs A)
 {
     extern __shared__ __align__(16) unsigned char smraw[];
     MSmem &sm = *reinterpret_cast<MSmem *>(smraw);
