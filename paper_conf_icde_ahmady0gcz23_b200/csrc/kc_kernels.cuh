@@ -48,7 +48,7 @@
 namespace kc {
 
 #ifndef KC_BLOCK
-#define KC_BLOCK 768
+#define KC_BLOCK 512
 #endif
 constexpr int kBlock = KC_BLOCK;
 constexpr int kWarps = kBlock / 32;
@@ -62,13 +62,13 @@ constexpr int kLCap = kBlock;        // local frontier capacity (entries; one pe
 constexpr int kLightLevelArcs = 4 << 20;
 constexpr int kHubLight = 32768, kSubLight = 32768, kPhaseLight = 262144;
 #ifndef KC_HUB
-#define KC_HUB 8192
+#define KC_HUB 32768
 #endif
 #ifndef KC_SUB
-#define KC_SUB 8192
+#define KC_SUB 32768
 #endif
 #ifndef KC_PHASE
-#define KC_PHASE 16384
+#define KC_PHASE 65536
 #endif
 constexpr int kHubHeavy = KC_HUB, kSubHeavy = KC_SUB, kPhaseHeavy = KC_PHASE;
 #ifndef KC_GSTAGE

@@ -260,3 +260,25 @@ def test_caller_workspace_and_stream():
         out = kc.kcore_decompose(r, c, workspace=ws)
     s.synchronize()
     assert np.array_equal(out.cpu().numpy(), ref)
+
+
+# ------------------------------------------------- degenerate / maximum shapes
+def test_dense_single_level_and_equal_hubs():
+    """K_2048 (one level, every arc walked in one HUB-sized cascade) and
+    K_{64,50000} (64 equal-degree hubs of 50,000 arcs, core 64 everywhere)."""
+    n = 2048
+    rp, ci = kcgen.csr_from_edges(n, itertools.combinations(range(n), 2))
+    for kw in (dict(), dict(bloom=False), dict(algo=kc.ALGO_HOSTLOOP)):
+        _check(rp, ci, np.full(n, n - 1, np.int32), **kw)
+    a, b = 64, 50_000
+    rp, ci = kcgen.csr_from_edges(a + b, [(i, a + j) for i in range(a) for j in range(b)])
+    for kw in (dict(), dict(l2_persist=False)):
+        _check(rp, ci, np.full(a + b, a, np.int32), **kw)
+
+
+def test_ragged_sizes():
+    """Vertex counts that are not multiples of any tile, warp or segment size."""
+    for n, seed in ((1, 1), (31, 2), (33, 3), (1023, 4), (12_345, 5), (148 * 512 + 7, 6)):
+        spec = kcgen.chunglu(n, 2.1, max(1, 6 * n), seed=seed)
+        rp, ci = kcgen.generate_host(spec)
+        _check(rp, ci)
