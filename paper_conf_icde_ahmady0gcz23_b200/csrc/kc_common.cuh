@@ -132,11 +132,12 @@ __device__ __forceinline__ uint32_t atom_or_claim(uint32_t *p, uint32_t bit, uin
 __device__ __forceinline__ int32_t ld_cg_i32(const int32_t *p) { return __ldcg(p); }
 __device__ __forceinline__ int64_t ld_cg_i64(const int64_t *p) { return __ldcg(p); }
 
-// Warm L2 with the adjacency row [b, e) of a vertex that was just claimed, so
+// Optionally warm L2 with the adjacency row [b, e) of a vertex that was just
+// claimed (measured: no gain on B200, off by default -- DESIGN.md §8), so
 // the next hop's colidx gathers hit L2: one TMA bulk prefetch of the whole
 // row (16-byte aligned, capped at KC_BULK_PF bytes), or the first line only.
 #ifndef KC_BULK_PF
-#define KC_BULK_PF 0
+#define KC_BULK_PF -1
 #endif
 __device__ __forceinline__ void prefetch_row(const int32_t *colidx, int64_t b, int64_t e)
 {
@@ -145,6 +146,8 @@ __device__ __forceinline__ void prefetch_row(const int32_t *colidx, int64_t b, i
     uintptr_t hi = (reinterpret_cast<uintptr_t>(colidx + e) + 15) & ~(uintptr_t)15;
     if (hi - lo > (uintptr_t)KC_BULK_PF) hi = lo + KC_BULK_PF;
     asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(lo), "r"((uint32_t)(hi - lo)) : "memory");
+#elif KC_BULK_PF < 0
+    (void)colidx; (void)b; (void)e;  // no prefetch (measurement variant)
 #else
     (void)e;
     asm volatile("prefetch.global.L2 [%0];" ::"l"(colidx + b));

@@ -101,6 +101,9 @@ constexpr int kTraceFields = 8;
 #ifndef KC_CF_LOCAL_MIN
 #define KC_CF_LOCAL_MIN 0
 #endif
+#ifndef KC_ROUTE4_INLINE
+#define KC_ROUTE4_INLINE 1
+#endif
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
 #endif
@@ -480,7 +483,12 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
 // the same decisions as four route_won calls, with ONE order/removed update,
 // ONE budget reservation and one local-list reservation for the whole warp
 // (the shared-memory atomics are a dependent chain on the hit path).
-__device__ __noinline__ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int32_t v1,
+#if KC_ROUTE4_INLINE
+__device__ __forceinline__
+#else
+__device__ __noinline__
+#endif
+void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int32_t v1,
                                         int32_t v2, int32_t v3, int32_t d0, int32_t d1, int32_t d2, int32_t d3,
                                         int64_t b0, int64_t b1, int64_t b2, int64_t b3, int nx, int &gcnt)
 {
