@@ -104,6 +104,9 @@ constexpr int kTraceFields = 8;
 #ifndef KC_ROUTE4_INLINE
 #define KC_ROUTE4_INLINE 1
 #endif
+#ifndef KC_SCAN_PIPE
+#define KC_SCAN_PIPE 1
+#endif
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
 #endif
@@ -896,16 +899,26 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const uint64_t pol = deg_policy();
     constexpr int CH = 32 * kScanItems;
-    for (int64_t off = lo + (int64_t)wib * CH; off < hi; off += (int64_t)kWarps * CH) {
-        int32_t vv[kScanItems], dd[kScanItems];
+    // software pipeline: the next chunk's alive entries are loaded while this
+    // chunk's degrees are in flight
+    int32_t vn[kScanItems];
+    auto load_chunk = [&](int64_t o) {
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
-            const int64_t idx = off + j * 32 + lane;
-            vv[j] = -1;
-            if (idx < hi) vv[j] = src ? ld_cg_i32(src + idx) : (int32_t)idx;
+            const int64_t idx = o + j * 32 + lane;
+            vn[j] = -1;
+            if (idx < hi) vn[j] = src ? ld_cg_i32(src + idx) : (int32_t)idx;
         }
+    };
+    load_chunk(lo + (int64_t)wib * CH);
+    for (int64_t off = lo + (int64_t)wib * CH; off < hi; off += (int64_t)kWarps * CH) {
+        int32_t vv[kScanItems], dd[kScanItems];
+        if (!KC_SCAN_PIPE && off != lo + (int64_t)wib * CH) load_chunk(off);
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) vv[j] = vn[j];
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) dd[j] = vv[j] >= 0 ? ld_deg(A.deg + vv[j], pol) : -1;
+        if (KC_SCAN_PIPE) load_chunk(off + (int64_t)kWarps * CH);
         unsigned wm = 0, km = 0;
 #pragma unroll
         for (int j = 0; j < kScanItems; j++) {
