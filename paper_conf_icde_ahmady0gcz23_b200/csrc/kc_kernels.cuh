@@ -203,6 +203,8 @@ struct Smem {
     int32_t removed;     // vertices removed by this CTA this phase (order not recorded)
     int32_t fit;         // unused
     int32_t kcur;        // scan: compaction cursor within the current segment
+    int32_t seg_cache[2];     // length of this CTA's own segment in alive[x], as it last wrote it
+    int32_t seg_cache_ok[2];  // (persistent kernel only; a k_phase launch starts without it)
     int32_t bud_hub, bud_sub, bud_phase, bud_pad;  // routing budgets of this phase
     unsigned long long scan_q2[kWarps];
     unsigned long long tot_q2, base_g, base_w;
@@ -882,7 +884,10 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
         const unsigned iso = __ballot_sync(kFull, d == 0);
         if ((threadIdx.x & 31) == 0) A.claimed[v0 >> 5] = iso;
     }
-    if (threadIdx.x == 0) { sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0; }
+    if (threadIdx.x == 0) {
+        sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
+        sm.seg_cache_ok[0] = sm.seg_cache_ok[1] = 0;
+    }
     block_min_atomic(sm, lmin, &A.S->min_next);
 }
 
@@ -996,7 +1001,8 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
         const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
         scan_range(A, c, sm, srcb, lo, hi, dst, lmin, gcnt);
     } else if (!solo) {
-        const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + bid);
+        // this CTA wrote its own segment's length at the last compaction
+        const int64_t len = sm.seg_cache_ok[c.src_sel] ? sm.seg_cache[c.src_sel] : ld_cg_i32(A.seg_len[c.src_sel] + bid);
         scan_range(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt);
     } else {
         for (int b = 0; b < A.nseg; b++) {
@@ -1007,6 +1013,8 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
     __syncthreads();
     if (threadIdx.x == 0 && dstb) {
         A.seg_len[c.dst_sel][dseg] = sm.kcur;
+        sm.seg_cache[c.dst_sel] = sm.kcur;
+        sm.seg_cache_ok[c.dst_sel] = solo ? 0 : 1;
         if (sm.kcur) atomicAdd(&A.S->alive_out, (unsigned long long)sm.kcur);
     }
 }
@@ -1335,6 +1343,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(const __grid_constant__ KAr
         sm.ctrl = A.S->pub;
         sm.bloom_on = 0;
         sm.bloom_level = -1;
+        sm.seg_cache_ok[0] = sm.seg_cache_ok[1] = 0;
     }
     __syncthreads();
     const Ctrl &c = sm.ctrl;
