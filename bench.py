@@ -269,7 +269,7 @@ def run_gpu(args):
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                      "algorithmic_bytes": b_min, "kernel_ms": kern_ms},
-        "gpu_launches": 3 * args.steps if (world == 1 and not args.force_mg) else None,  # init_state, persistent, l2_release
+        "gpu_launches": int(sum(s.launches for s in stats)),  # counted by the library, timed steps only
         "e2e": e2e,
         "clocks": clk,
         "stats": {"levels": st.levels, "phases": st.phases, "barriers": st.barriers, "scanned": st.scanned,

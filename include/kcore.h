@@ -121,7 +121,8 @@ typedef struct {
     int32_t block_threads;
     int32_t trace_len;     /* trace records written (see kcore_options.trace_out)    */
     double kernel_ms;      /* device time of the decomposition kernel(s) (CUDA events) */
-    int64_t reserved[3];
+    int64_t launches;      /* kernels this call launched                              */
+    int64_t reserved[2];
 } kcore_stats;
 
 /* Core decomposition on one GPU (north-star signature).  All array pointers

@@ -74,7 +74,7 @@ class _Stats(ctypes.Structure):
         ("compactions", ctypes.c_int64), ("hub_arcs", ctypes.c_int64), ("kmax", ctypes.c_int32),
         ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
         ("trace_len", ctypes.c_int32), ("kernel_ms", ctypes.c_double),
-        ("reserved", ctypes.c_int64 * 3),
+        ("launches", ctypes.c_int64), ("reserved", ctypes.c_int64 * 2),
     ]
 
 
@@ -93,12 +93,13 @@ class Stats:
     block_threads: int
     kernel_ms: float
     trace_len: int = 0
+    launches: int = 0
 
     @classmethod
     def _from(cls, s: _Stats) -> "Stats":
         return cls(s.levels, s.phases, s.solo_phases, s.barriers, s.scanned, s.arcs_walked,
                    s.compactions, s.hub_arcs, s.kmax, s.grid_blocks, s.block_threads, s.kernel_ms,
-                   s.trace_len)
+                   s.trace_len, s.launches)
 
 
 _lib = None

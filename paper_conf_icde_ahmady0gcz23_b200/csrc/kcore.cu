@@ -209,6 +209,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     int32_t *d_phase = nullptr;
     int64_t l2_lines = 0;
+    int64_t hl_launches = 0;
     const char *l2_base = nullptr;
     State hS;
     Carve cv;
@@ -300,9 +301,11 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaMallocAsync((void **)&d_phase, sizeof(int32_t), st));
         int32_t ph = PH_INIT;
         int guard = 0;
+        hl_launches = 1;  // k_init_state
         while (ph != PH_DONE) {
             k_phase<<<grid, kBlock, smem, st>>>(A);
             k_leader<<<1, 1, 0, st>>>(A, d_phase);
+            hl_launches += 2;
             KC_CUDA(cudaGetLastError());
             KC_CUDA(cudaMemcpyAsync(&ph, d_phase, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
             KC_CUDA(cudaStreamSynchronize(st));
@@ -337,6 +340,7 @@ launched:
         stats->block_threads = kBlock;
         stats->trace_len = (int32_t)hS.trace_n;
         stats->kernel_ms = ms;
+        stats->launches = algo == KCORE_ALGO_PERSISTENT ? 2 + (l2_lines > 0 ? 1 : 0) : hl_launches;
     }
 done:
     if (d_phase) cudaFreeAsync(d_phase, st);

@@ -369,7 +369,7 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
         recv(L, std::vector<unsigned long long>(P)), soff(L, std::vector<unsigned long long>(P + 1)),
         roff(L, std::vector<unsigned long long>(P + 1));
     std::vector<int64_t> fcnt(L, 0);
-    int64_t levels = 0, subrounds = 0, exchanged = 0;
+    int64_t levels = 0, subrounds = 0, exchanged = 0, launches = 0;
     int kmax = 0;
 
     // deg init and the first k
@@ -377,6 +377,7 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
     for (int r = 0; r < L; r++) {
         k_mg_reset<<<1, 64, 0, st>>>(R[r].ctl, P);
         if (R[r].nl) k_mg_init<<<grid_for(R[r].nl), kMgBlock, 0, st>>>(R[r], &R[r].ctl->min_next);
+        launches += 1 + (R[r].nl ? 1 : 0);
         MG_CK(cudaGetLastError());
         MG_CK(cudaMemcpyAsync(&hc[r], R[r].ctl, sizeof(MgCtl), cudaMemcpyDeviceToHost, st));
     }
@@ -395,6 +396,7 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
         for (int r = 0; r < L; r++) {
             k_mg_reset<<<1, 64, 0, st>>>(R[r].ctl, P);
             if (R[r].nl) k_mg_scan<<<grid_for(R[r].nl), kMgBlock, 0, st>>>(R[r], k);
+            launches += 1 + (R[r].nl ? 1 : 0);
             MG_CK(cudaGetLastError());
             MG_CK(cudaMemcpyAsync(&hc[r], R[r].ctl, sizeof(MgCtl), cudaMemcpyDeviceToHost, st));
         }
@@ -418,7 +420,9 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
                 if (fcnt[r]) {
                     k_mg_count<false><<<grid_for(fcnt[r] * 32), kMgBlock, 0, st>>>(R[r], O, fcnt[r], self0 + r);
                     k_mg_count<true><<<grid_for(fcnt[r] * kMgBlock), kMgBlock, 0, st>>>(R[r], O, fcnt[r], self0 + r);
+                    launches += 2;
                 }
+                launches++;
                 MG_CK(cudaGetLastError());
                 MG_CK(cudaMemcpyAsync(&hc[r], R[r].ctl, sizeof(MgCtl), cudaMemcpyDeviceToHost, st));
             }
@@ -449,13 +453,17 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
                 if (fcnt[r]) {
                     k_mg_fill<false><<<grid_for(fcnt[r] * 32), kMgBlock, 0, st>>>(R[r], O, S, fcnt[r], self0 + r, k);
                     k_mg_fill<true><<<grid_for(fcnt[r] * kMgBlock), kMgBlock, 0, st>>>(R[r], O, S, fcnt[r], self0 + r, k);
+                    launches += 2;
                 }
                 MG_CK(cudaGetLastError());
             }
             MG_RC(T.exchange_payload(R, send, soff, recv, roff));
             for (int r = 0; r < L; r++) {
                 const int64_t cnt = (int64_t)roff[r][P];
-                if (cnt) k_mg_apply<<<grid_for(cnt), kMgBlock, 0, st>>>(R[r], cnt, O.start[self0 + r], k);
+                if (cnt) {
+                    k_mg_apply<<<grid_for(cnt), kMgBlock, 0, st>>>(R[r], cnt, O.start[self0 + r], k);
+                    launches++;
+                }
                 MG_CK(cudaGetLastError());
                 MG_CK(cudaMemcpyAsync(&hc[r], R[r].ctl, sizeof(MgCtl), cudaMemcpyDeviceToHost, st));
             }
@@ -479,6 +487,7 @@ int mg_drive(std::vector<RankView> &R, const Owners &O, int self0, Transport &T,
         stats->phases = subrounds;
         stats->kmax = kmax;
         stats->hub_arcs = exchanged;  // remote decrements sent by the local ranks
+        stats->launches = launches;
     }
     return KCORE_OK;
 }

@@ -377,6 +377,7 @@ extern "C" int kcore_mpm(const int64_t *rowptr, const int32_t *colidx, int64_t n
             stats->grid_blocks = grid;
             stats->block_threads = kB;
             stats->kernel_ms = ms;
+            stats->launches = 2;  // k_mpm_init, k_mpm
         }
     }
     cudaFreeAsync(ws, st);
