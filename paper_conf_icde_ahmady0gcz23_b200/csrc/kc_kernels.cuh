@@ -101,6 +101,9 @@ constexpr int kTraceFields = 8;
 #ifndef KC_CF_LOCAL_MIN
 #define KC_CF_LOCAL_MIN 0
 #endif
+#ifndef KC_HITS_INLINE
+#define KC_HITS_INLINE 0
+#endif
 #ifndef KC_ROUTE4_INLINE
 #define KC_ROUTE4_INLINE 1
 #endif
@@ -601,7 +604,12 @@ __device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
 // --------------------------------------------------------- arc walking
 // Hits of one batch (u reached k): claim, fetch row bounds, prefetch the
 // row's first line for the next hop, route.  Out of line: rare path.
-__device__ __noinline__ void handle_hits(const KArgs &A, Smem &sm, int k, int nx, int u0, int u1, int u2, int u3,
+#if KC_HITS_INLINE
+__device__ __forceinline__
+#else
+__device__ __noinline__
+#endif
+void handle_hits(const KArgs &A, Smem &sm, int k, int nx, int u0, int u1, int u2, int u3,
                                          unsigned hm, int &gcnt)
 {
     const int wib = threadIdx.x >> 5;
