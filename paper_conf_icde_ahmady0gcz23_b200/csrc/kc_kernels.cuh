@@ -102,7 +102,7 @@ constexpr int kTraceFields = 8;
 #define KC_CF_LOCAL_MIN 0
 #endif
 #ifndef KC_HITS_INLINE
-#define KC_HITS_INLINE 0
+#define KC_HITS_INLINE 1
 #endif
 #ifndef KC_ROUTE4_INLINE
 #define KC_ROUTE4_INLINE 1
