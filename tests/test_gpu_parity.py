@@ -282,3 +282,24 @@ def test_ragged_sizes():
         spec = kcgen.chunglu(n, 2.1, max(1, 6 * n), seed=seed)
         rp, ci = kcgen.generate_host(spec)
         _check(rp, ci)
+
+
+@pytest.mark.slow
+def test_more_than_2_31_arcs_closed_form():
+    """64-bit arc offsets: K_{48, 23M} has 2.2e9 arcs (> 2^31) and 48 hubs of
+    23M arcs each; every core number is min(a, b) = 48 (closed form)."""
+    a, b = 48, 23_000_000
+    n = a + b
+    dev = torch.device(DEV)
+    deg = torch.cat([torch.full((a,), b, dtype=torch.int64, device=dev),
+                     torch.full((b,), a, dtype=torch.int64, device=dev)])
+    rowptr = torch.zeros(n + 1, dtype=torch.int64, device=dev)
+    rowptr[1:] = torch.cumsum(deg, 0)
+    assert int(rowptr[-1]) > (1 << 31)
+    colidx = torch.cat([torch.arange(a, n, dtype=torch.int32, device=dev).repeat(a),
+                        torch.arange(a, dtype=torch.int32, device=dev).repeat(b)])
+    del deg
+    core = kc.kcore_decompose(rowptr, colidx)
+    assert bool((core == a).all())
+    del core
+    torch.cuda.empty_cache()
