@@ -197,8 +197,9 @@ int kcore_kcore_subgraph(const int64_t *rowptr, const int32_t *colidx, const int
  * until an iteration changes nothing (then a = core) or `max_iters`
  * iterations have run (max_iters < 0: no limit).  DEVICE rowptr/colidx/a_out
  * (int32[n], the last iterate).  *iters_out (HOST, may be NULL) = iterations
- * that changed at least one value.  One persistent cooperative kernel;
- * scratch (about 24 n bytes) is allocated stream-ordered.  Synchronises
+ * that changed at least one value.  One persistent cooperative kernel with
+ * exact support counters (only vertices that will change are recomputed);
+ * scratch (about 32 n bytes) is allocated stream-ordered.  Synchronises
  * `stream`.  stats (may be NULL): levels = phases = iterations, scanned =
  * sum of active-set sizes, arcs_walked = arcs gathered, kernel_ms. */
 int kcore_mpm(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m, int32_t *a_out,

@@ -10,19 +10,25 @@
 // with the oracle (oracle_mpm).
 //
 // One persistent cooperative kernel per call (no host round trip per
-// iteration).  Per iteration t:
-//   A1  warps take the active vertices; a vertex with <= 128 arcs keeps its
-//       neighbours' (capped) estimates in registers and binary-searches h
-//       with ballot counts; bigger vertices go to a per-iteration list.
-//   A2  CTAs take the big vertices one at a time: a 1024-bin histogram of the
-//       capped estimates over the candidate range [lo, hi] (per-warp
-//       sub-histograms in shared memory, so equal estimates do not serialise
-//       on one bin), a suffix count picks the bin holding h, and the range
-//       shrinks 1024x per pass (<= 3 passes for any degree < 2^30).
-//   Every vertex whose estimate dropped is recorded, and its neighbours are
-//   stamped active for t+1 (a vertex whose neighbours did not change cannot
-//   change: the active set is exact for the Jacobi iteration).
-//   C   commit the new estimates of the changed vertices.
+// iteration), with exact SUPPORT COUNTERS: cnt(v) = |{u in N(v) : a(u) >= a(v)}|.
+// v keeps its estimate at the next iteration iff cnt(v) >= a(v), so the next
+// active set is exactly the set of vertices that WILL change -- hubs are no
+// longer re-read whenever a neighbour moves.  Per iteration t:
+//   A1  warps take the active vertices with <= 128 arcs: the neighbours'
+//       capped estimates a_{t-1} stay in registers; a ballot-count binary
+//       search gives h = max{h : N(h) >= h} and N(h); bigger vertices are
+//       deferred to a list.
+//   A2  CTAs take the big vertices: one counting pass decides "unchanged"
+//       (t = 1 only; later every active vertex changes), else a 1024-bin
+//       histogram over [lo, hi] (per-warp sub-histograms in shared memory) and
+//       a warp suffix search shrink the range 1024x per pass.
+//       Every computed vertex stores cnt(v) = N_{t-1}(h); a changed one also
+//       stores a_new(v) = h and the stamp cstamp(v) = t.
+//   B   every changed x tells each neighbour u whose support it withdraws:
+//       if a_{t-1}(x) >= a_t(u) > a_t(x) then cnt(u) -= 1; the decrement that
+//       takes cnt(u) from a_t(u) to a_t(u)-1 activates u for t+1 (exactly
+//       once).  After B, cnt(u) = |{x : a_t(x) >= a_t(u)}| for every u.
+//   C   commit a_t(x) for the changed vertices.
 // Estimates never increase (a_{t+1} <= a_t, induction on the monotone
 // h-index), so h is searched in [0, min(a_t(v), deg(v))] only.
 #include "kcore.h"
@@ -44,8 +50,9 @@ constexpr int kBins = 1024;
 
 struct MState {
     unsigned long long act_len[2];      // active list lengths, by iteration parity
-    unsigned long long chg_len[2];      // changed vertices
+    unsigned long long chg_len[2];      // changed vertices with <= kSmall arcs
     unsigned long long big_len[2];      // big active vertices
+    unsigned long long cbig_len[2];     // changed vertices with > kSmall arcs
     unsigned long long iters;           // iterations that changed something
     unsigned long long processed;       // sum of active-set sizes (statistics)
     unsigned long long arcs;            // arcs gathered (statistics)
@@ -56,9 +63,11 @@ struct MArgs {
     const int32_t *colidx;
     int32_t *a;        // current iterate (= a_out)
     int32_t *a_new;    // next values of the changed vertices
-    int32_t *stamp;    // last iteration a vertex was activated for
+    int32_t *cnt;      // support counters
+    int32_t *cstamp;   // iteration at which a vertex last changed
     int32_t *act[2];   // active lists
-    int32_t *chg;      // changed vertices of this iteration
+    int32_t *chg;      // changed vertices of this iteration (small)
+    int32_t *cbig;     // changed vertices of this iteration (big)
     int32_t *big;      // big active vertices of this iteration
     MState *S;
     int64_t n;
@@ -91,21 +100,22 @@ __device__ __forceinline__ void warp_append(bool p, int32_t v, int32_t *list, un
     if (p) list[base + __popc(b & lanemask_lt())] = v;
 }
 
-// Activate, for iteration t+1, the neighbours u of a vertex whose estimate
-// dropped to h at iteration t (warp, arcs [b0+lane0, e) step `step`).  Only
-// neighbours with a_{t-1}(u) > h: u's next value is the h-index of its
-// neighbours' estimates capped at a_t(u) <= a_{t-1}(u), so a neighbour whose
-// new value is still >= a_{t-1}(u) cannot change it -- the filter keeps the
-// active set exact for the Jacobi iteration.
-__device__ __forceinline__ void activate(const MArgs &A, int64_t b0, int64_t e, int64_t step, int t1, int32_t h)
+// B: x changed at iteration t from ax = a_{t-1}(x) to hx = a_t(x); withdraw
+// its support from the neighbours u with ax >= a_t(u) > hx (warp, arcs
+// [b0+lane0, e) step `step`).  The decrement that takes cnt(u) from a_t(u) to
+// a_t(u)-1 activates u for iteration t+1.
+__device__ __forceinline__ void notify(const MArgs &A, int64_t b0, int64_t e, int64_t step, int t, int32_t ax,
+                                       int32_t hx)
 {
+    const int t1 = t + 1;
     for (int64_t x0 = b0; x0 < e; x0 += step) {
         const int64_t x = x0 + (threadIdx.x & 31);
         bool p = false;
         int32_t u = 0;
         if (x < e) {
             u = __ldg(A.colidx + x);
-            p = __ldcg(A.a + u) > h && atomicExch(A.stamp + u, t1) != t1;
+            const int32_t au = __ldcg(A.cstamp + u) == t ? __ldcg(A.a_new + u) : __ldcg(A.a + u);
+            if (ax >= au && au > hx) p = atomicSub(A.cnt + u, 1) == au;
         }
         warp_append(p, u, A.act[t1 & 1], &A.S->act_len[t1 & 1]);
     }
@@ -122,28 +132,33 @@ __device__ __forceinline__ void small_vertex(const MArgs &A, int32_t v, int64_t 
         const int64_t i = r * 32 + lane;
         x[r] = i < d ? min(__ldcg(A.a + __ldg(A.colidx + b + i)), c) : -1;
     }
-    int lo = 0, hi = (int)min((int64_t)c, d);
+    int lo = 0, hi = (int)min((int64_t)c, d), nlo = (int)d;  // nlo = N(lo)
     while (lo < hi) {
         const int mid = (lo + hi + 1) >> 1;
         int cnt = 0;
 #pragma unroll
         for (int r = 0; r < kSmall / 32; r++) cnt += __popc(__ballot_sync(kFull, x[r] >= mid));
-        if (cnt >= mid) lo = mid; else hi = mid - 1;
+        if (cnt >= mid) { lo = mid; nlo = cnt; } else hi = mid - 1;
     }
     const bool ch = lo != c;
-    if (ch && lane == 0) A.a_new[v] = lo;
+    if (lane == 0) {
+        A.cnt[v] = nlo;
+        if (ch) { A.a_new[v] = lo; A.cstamp[v] = t; }
+    }
     warp_append(ch && lane == 0, v, A.chg, &A.S->chg_len[t & 1]);
-    if (ch) activate(A, b, b + d, 32, t + 1, lo);
 }
 
 // A2: the whole CTA, vertex v with d > kSmall arcs
-__device__ void big_vertex(const MArgs &A, MSmem &sm, int32_t v, int t)
+__device__ void big_vertex(const MArgs &A, MSmem &sm, int32_t v, int t)  // t: iteration
 {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     const int64_t b = __ldg(A.rowptr + v), e = __ldg(A.rowptr + v + 1), d = e - b;
     const int32_t c = __ldcg(A.a + v);
     int64_t lo = 0, hi = min((int64_t)c, d);  // h in [lo, hi]; |{x >= lo}| >= lo holds
-    {
+    int32_t nlo = (int32_t)d;                  // N(lo)
+    if (t > 1) {
+        hi = hi - 1;  // an active vertex always drops (its support fell below a(v))
+    } else {
         // most active big vertices keep their estimate: one counting pass
         // decides N(hi) >= hi without building a histogram
         int64_t cnt = 0;
@@ -156,9 +171,10 @@ __device__ void big_vertex(const MArgs &A, MSmem &sm, int32_t v, int t)
             int64_t s = 0;
             for (int q = 0; q < kW; q++) s += sm.wsum[q];
             sm.bcast[0] = s >= hi ? 1 : 0;
+            sm.bcast[1] = (int32_t)s;
         }
         __syncthreads();
-        if (sm.bcast[0]) lo = hi;
+        if (sm.bcast[0]) { lo = hi; nlo = sm.bcast[1]; }
         else hi = hi - 1;
         __syncthreads();
     }
@@ -214,25 +230,36 @@ __device__ void big_vertex(const MArgs &A, MSmem &sm, int32_t v, int t)
             const unsigned bl = __ballot_sync(kFull, best >= 0);
             const int src = 31 - __clz(bl);
             const int jb = __shfl_sync(kFull, best, src);
-            if (lane == 0) sm.bcast[0] = jb;
+            // N at the chosen bin start: recompute the suffix there
+            int64_t nb = 0;
+            if (lane == src) {
+                int64_t sf = sm.wsum[kW] + inc - part;
+                for (int q = per - 1; q >= 0; q--) {
+                    sf += sm.tot[lane * per + q];
+                    if (lane * per + q == jb) { nb = sf; break; }
+                }
+            }
+            nb = __shfl_sync(kFull, nb, src);
+            if (lane == 0) { sm.bcast[0] = jb; sm.bcast[1] = (int32_t)nb; }
         }
         __syncthreads();
         const int jb = sm.bcast[0];
+        nlo = sm.bcast[1];
         const int64_t nlo = lo + (int64_t)jb * wd;
         hi = min(hi, nlo + wd - 1);
         lo = nlo;
         __syncthreads();
     }
     const int32_t h = (int32_t)lo;
-    if (h != c) {
-        if (threadIdx.x == 0) {
+    if (threadIdx.x == 0) {
+        A.cnt[v] = nlo;
+        if (h != c) {
             A.a_new[v] = h;
-            const unsigned long long p = atomicAdd(&A.S->chg_len[t & 1], 1ULL);
-            A.chg[p] = v;
+            A.cstamp[v] = t;
+            A.cbig[atomicAdd(&A.S->cbig_len[t & 1], 1ULL)] = v;
         }
-        // activate neighbours with every warp of the CTA
-        activate(A, b + (int64_t)w * 32, e, (int64_t)kB, t + 1, h);
     }
+    __syncthreads();
 }
 
 __global__ void __launch_bounds__(kB, 1) k_mpm(const __grid_constant__ MArgs A)
@@ -247,13 +274,7 @@ __global__ void __launch_bounds__(kB, 1) k_mpm(const __grid_constant__ MArgs A)
     unsigned long long processed = 0, arcs = 0;
     for (int t = 1;; t++) {
         if (A.max_iters >= 0 && t > A.max_iters) break;
-        // reset the counters of the parity this iteration will fill next
-        if (blockIdx.x == 0 && threadIdx.x == 0) {
-            S->act_len[(t + 1) & 1] = 0;
-            S->chg_len[t & 1] = 0;  // read by every CTA only after the syncs of iteration t-2
-            S->big_len[t & 1] = 0;
-        }
-        grid.sync();
+        // (counters of parity t were reset in phase C of iteration t-1 / by k_mpm_init)
         const int64_t len = (t == 1) ? A.n : (int64_t)__ldcg(&S->act_len[t & 1]);
         const int32_t *act = A.act[t & 1];
         // A1: small vertices by warps, big ones deferred
@@ -272,14 +293,37 @@ __global__ void __launch_bounds__(kB, 1) k_mpm(const __grid_constant__ MArgs A)
         const int64_t nbig = (int64_t)__ldcg(&S->big_len[t & 1]);
         for (int64_t i = blockIdx.x; i < nbig; i += gridDim.x) big_vertex(A, sm, __ldcg(A.big + i), t);
         grid.sync();
-        // C: commit (Jacobi: every read of iterate t-1 happened before the sync)
         const int64_t nchg = (int64_t)__ldcg(&S->chg_len[t & 1]);
-        if (nchg == 0) break;
-        for (int64_t i = (int64_t)blockIdx.x * kB + threadIdx.x; i < nchg; i += (int64_t)gridDim.x * kB) {
-            const int32_t v = __ldcg(A.chg + i);
-            A.a[v] = __ldcg(A.a_new + v);
+        const int64_t ncbig = (int64_t)__ldcg(&S->cbig_len[t & 1]);
+        if (nchg + ncbig == 0) break;
+        // B: changed vertices withdraw their support (small ones by warps, big ones by CTAs)
+        for (int64_t i = gw; i < nchg; i += nw) {
+            const int32_t x = __ldcg(A.chg + i);
+            const int64_t b = __ldg(A.rowptr + x), e = __ldg(A.rowptr + x + 1);
+            notify(A, b, e, 32, t, __ldcg(A.a + x), __ldcg(A.a_new + x));
+            if (lane == 0) arcs += e - b;
         }
-        if (blockIdx.x == 0 && threadIdx.x == 0) S->iters = (unsigned long long)t;
+        for (int64_t i = blockIdx.x; i < ncbig; i += gridDim.x) {
+            const int32_t x = __ldcg(A.cbig + i);
+            const int64_t b = __ldg(A.rowptr + x), e = __ldg(A.rowptr + x + 1);
+            notify(A, b + (int64_t)(threadIdx.x >> 5) * 32, e, (int64_t)kB, t, __ldcg(A.a + x), __ldcg(A.a_new + x));
+            if (threadIdx.x == 0) arcs += e - b;
+        }
+        grid.sync();
+        // C: commit (Jacobi: every read of iterate t-1 happened before the syncs);
+        // reset the counters iteration t+1 will fill (their last readers are done)
+        for (int64_t i = (int64_t)blockIdx.x * kB + threadIdx.x; i < nchg + ncbig; i += (int64_t)gridDim.x * kB) {
+            const int32_t x = i < nchg ? __ldcg(A.chg + i) : __ldcg(A.cbig + (i - nchg));
+            A.a[x] = __ldcg(A.a_new + x);
+        }
+        if (blockIdx.x == 0 && threadIdx.x == 0) {
+            S->iters = (unsigned long long)t;
+            S->act_len[t & 1] = 0;  // input of iteration t: read at its start
+            S->chg_len[(t + 1) & 1] = 0;
+            S->big_len[(t + 1) & 1] = 0;
+            S->cbig_len[(t + 1) & 1] = 0;
+        }
+        grid.sync();
     }
     if (lane == 0 && processed) {
         atomicAdd(&S->processed, processed);
@@ -287,17 +331,18 @@ __global__ void __launch_bounds__(kB, 1) k_mpm(const __grid_constant__ MArgs A)
     }
 }
 
-__global__ void k_mpm_init(const int64_t *rowptr, int64_t n, int32_t *a, int32_t *stamp, MState *S)
+__global__ void k_mpm_init(const int64_t *rowptr, int64_t n, int32_t *a, int32_t *cstamp, MState *S)
 {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n; v += stride) {
         a[v] = (int32_t)(rowptr[v + 1] - rowptr[v]);
-        stamp[v] = 0;
+        cstamp[v] = 0;
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         S->act_len[0] = S->act_len[1] = 0;
         S->chg_len[0] = S->chg_len[1] = 0;
         S->big_len[0] = S->big_len[1] = 0;
+        S->cbig_len[0] = S->cbig_len[1] = 0;
         S->iters = S->processed = S->arcs = 0;
     }
 }
@@ -327,7 +372,7 @@ extern "C" int kcore_mpm(const int64_t *rowptr, const int32_t *colidx, int64_t n
         return KCORE_EUNSUPPORTED;
     const int grid = sms * occ;
     const size_t nn = (size_t)n;
-    const size_t bytes = al(sizeof(MState)) + 6 * al(sizeof(int32_t) * nn);
+    const size_t bytes = al(sizeof(MState)) + 8 * al(sizeof(int32_t) * nn);
     char *ws = nullptr;
     int rc = KCORE_OK;
     cudaEvent_t e0 = nullptr, e1 = nullptr;
@@ -339,10 +384,12 @@ extern "C" int kcore_mpm(const int64_t *rowptr, const int32_t *colidx, int64_t n
         char *p = ws;
         A.S = (MState *)p; p += al(sizeof(MState));
         A.a_new = (int32_t *)p; p += al(sizeof(int32_t) * nn);
-        A.stamp = (int32_t *)p; p += al(sizeof(int32_t) * nn);
+        A.cnt = (int32_t *)p; p += al(sizeof(int32_t) * nn);
+        A.cstamp = (int32_t *)p; p += al(sizeof(int32_t) * nn);
         A.act[0] = (int32_t *)p; p += al(sizeof(int32_t) * nn);
         A.act[1] = (int32_t *)p; p += al(sizeof(int32_t) * nn);
         A.chg = (int32_t *)p; p += al(sizeof(int32_t) * nn);
+        A.cbig = (int32_t *)p; p += al(sizeof(int32_t) * nn);
         A.big = (int32_t *)p;
     }
     A.rowptr = rowptr;
@@ -356,7 +403,7 @@ extern "C" int kcore_mpm(const int64_t *rowptr, const int32_t *colidx, int64_t n
         cudaEventCreate(&e1);
         cudaEventRecord(e0, st);
     }
-    k_mpm_init<<<std::min<int64_t>((n + 255) / 256, (int64_t)sms * 8), 256, 0, st>>>(rowptr, n, a_out, A.stamp, A.S);
+    k_mpm_init<<<std::min<int64_t>((n + 255) / 256, (int64_t)sms * 8), 256, 0, st>>>(rowptr, n, a_out, A.cstamp, A.S);
     e = cudaGetLastError();
     if (e == cudaSuccess) e = cudaLaunchCooperativeKernel((const void *)k_mpm, dim3(grid), dim3(kB), args, smem, st);
     if (e == cudaSuccess && stats) e = cudaEventRecord(e1, st);
@@ -371,7 +418,7 @@ extern "C" int kcore_mpm(const int64_t *rowptr, const int32_t *colidx, int64_t n
             cudaEventElapsedTime(&ms, e0, e1);
             stats->levels = (int64_t)hS.iters;
             stats->phases = (int64_t)hS.iters;
-            stats->barriers = 3 * ((int64_t)hS.iters + 1);
+            stats->barriers = 4 * (int64_t)hS.iters + 2;
             stats->scanned = (int64_t)hS.processed;
             stats->arcs_walked = (int64_t)hS.arcs;
             stats->grid_blocks = grid;
