@@ -23,6 +23,6 @@ print(json.dumps(out))
 ''' % (names, KWS)
 for v in VAR:
     env = dict(os.environ, KCORE_LIB=os.path.abspath(v))
-    p = subprocess.run([sys.executable, "-c", CODE], env=env, capture_output=True, text=True, timeout=600)
+    p = subprocess.run([sys.executable, "-c", CODE], env=env, capture_output=True, text=True, timeout=240)
     res = p.stdout.strip().splitlines()[-1] if p.stdout.strip() else p.stderr[-300:]
     print(f"{os.path.basename(v):12s} {res}", flush=True)
