@@ -303,3 +303,22 @@ def test_more_than_2_31_arcs_closed_form():
     assert bool((core == a).all())
     del core
     torch.cuda.empty_cache()
+
+
+def test_concurrent_calls_on_two_streams():
+    """Two decompositions in flight on different streams (each call owns its
+    workspace and control state; cooperative launches serialise on the SMs)."""
+    g1 = kcgen.generate_host(kcgen.rmat(14, 16, seed=21))
+    g2 = kcgen.generate_host(kcgen.chunglu(20000, 2.1, 200000, seed=22))
+    refs = [oracle.bz_core(*g1), oracle.bz_core(*g2)]
+    devs = [_to_dev(*g1), _to_dev(*g2)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    for rep in range(5):
+        outs = []
+        for (r, c), s in zip(devs, streams):
+            with torch.cuda.stream(s):
+                outs.append(kc.kcore_decompose(r, c))
+        for s in streams:
+            s.synchronize()
+        for o, ref in zip(outs, refs):
+            assert np.array_equal(o.cpu().numpy(), ref), rep
