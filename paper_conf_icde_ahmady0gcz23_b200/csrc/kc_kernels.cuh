@@ -876,27 +876,44 @@ __device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &
 __device__ void phase_init(const KArgs &A, Smem &sm)
 {
     int lmin = INT_MAX;
+    unsigned niso = 0;
+    const int lane = threadIdx.x & 31;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    // claim bits start set exactly for the isolated vertices (removed at
-    // k = 0 without a claim): a warp covers 32 consecutive, aligned ids
+    if (threadIdx.x == 0) sm.removed = 0;
+    __syncthreads();
+    // The 0-shell is the isolated vertices: nothing can reach them, so
+    // they are removed here -- claim bit set, core 0, counted as removed -- and
+    // the first level is the smallest positive degree (no full scan at k = 0).
+    // A warp covers 32 consecutive, aligned ids (one claim-bit word).
     static_assert(kBlock % 32 == 0, "warps cover aligned 32-vertex words");
-    for (int64_t v0 = tid - (threadIdx.x & 31); v0 < A.n; v0 += stride) {
-        const int64_t v = v0 + (threadIdx.x & 31);
+    for (int64_t v0 = tid - lane; v0 < A.n; v0 += stride) {
+        const int64_t v = v0 + lane;
         int32_t d = -1;
         if (v < A.n) {
             d = (int32_t)(ld_ro_i64(A.rowptr + v + 1) - ld_ro_i64(A.rowptr + v));
             A.deg[v] = d;
-            lmin = min(lmin, d);
+            if (d > 0) lmin = min(lmin, d);
+            else A.core[v] = 0;
         }
         const unsigned iso = __ballot_sync(kFull, d == 0);
-        if ((threadIdx.x & 31) == 0) A.claimed[v0 >> 5] = iso;
+        if (lane == 0) A.claimed[v0 >> 5] = iso;
+        if (iso && A.order) {  // peel order requested: the 0-shell comes first
+            unsigned long long base = 0;
+            if (lane == 0) base = atomicAdd(&A.S->ord_tail, (unsigned long long)__popc(iso));
+            base = __shfl_sync(kFull, base, 0);
+            if (d == 0) A.order[base + __popc(iso & lanemask_lt())] = (int32_t)v;
+        } else if (iso && lane == 0) {
+            niso += __popc(iso);
+        }
     }
+    if (lane == 0 && niso) atomicAdd(&sm.removed, (int)niso);
     if (threadIdx.x == 0) {
         sm.bloom_on = 0; sm.bloom_level = -1; sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
         sm.seg_cache_ok[0] = sm.seg_cache_ok[1] = 0;
     }
-    block_min_atomic(sm, lmin, &A.S->min_next);
+    block_min_atomic(sm, lmin, &A.S->min_next);  // (ends with __syncthreads)
+    if (threadIdx.x == 0 && sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
 }
 
 // ------------------------------------------------------------------ LEVEL
@@ -1122,7 +1139,12 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
     int next_k = 0;
     bool new_level = false;
     if (c.phase == PH_INIT) {
-        next_k = (c.level_min == INT_MAX) ? 0 : c.level_min;
+        if (removed > 0) { c.st_levels = 1; c.st_kmax = 0; }  // the 0-shell, removed by INIT
+        if (removed >= p.n) {  // nothing but isolated vertices
+            c.phase = PH_DONE;
+            return;
+        }
+        next_k = c.level_min;  // smallest positive degree
         c.level_min = INT_MAX;
         c.level = -1;
         new_level = true;
