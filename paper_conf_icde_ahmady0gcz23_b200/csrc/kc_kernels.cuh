@@ -110,6 +110,9 @@ constexpr int kTraceFields = 8;
 #ifndef KC_SCAN_PIPE
 #define KC_SCAN_PIPE 1
 #endif
+#ifndef KC_COMPACT_D
+#define KC_COMPACT_D 32 // compact the alive list once >= 1/KC_COMPACT_D of it is dead
+#endif
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
 #endif
@@ -1191,7 +1194,7 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
     if (new_level) {
         const int64_t live = p.n - removed;
         const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
-        const bool compact = live * 8 < src_len * 7;  // >= 1/8 of the scan source is dead
+        const bool compact = live * KC_COMPACT_D < src_len * (KC_COMPACT_D - 1);  // >= 1/D of the source is dead
         c.phase = PH_LEVEL;
         c.k = next_k;
         c.level++;
