@@ -139,7 +139,10 @@ int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, int64_t n, 
  * decomposes, copies core_out device->host, and synchronises `stream` before
  * returning.  Host buffers should be pinned for full PCIe bandwidth.
  * Device memory for the graph and scratch is allocated stream-ordered and
- * freed before return. */
+ * freed before return.  The first call sets the release threshold of the
+ * device's default memory pool to "never" (device-wide, cudaMallocAsync users
+ * only), so repeated calls reuse the pool's pages instead of re-mapping
+ * gigabytes each time. */
 int kcore_decompose_host(const int64_t *rowptr_host, const int32_t *colidx_host, int64_t n,
                          int64_t m, int32_t *core_out_host, void *stream,
                          const kcore_options *opt, kcore_stats *stats);

@@ -356,6 +356,28 @@ extern "C" int kcore_decompose(const int64_t *rowptr, const int32_t *colidx, int
     return kcore_decompose_ex(rowptr, colidx, n, m, core_out, stream, nullptr, nullptr);
 }
 
+namespace {
+// The host entry point moves gigabytes per call through stream-ordered
+// allocations; by default the pool returns freed memory to the driver at every
+// synchronisation, so each call would re-map its buffers.  Keep what the pool
+// holds (cudaMemPoolAttrReleaseThreshold on the device's default pool, set
+// once; torch's caching allocator does not use this pool).
+void keep_pool_warm()
+{
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDev) return;
+    static bool done[kMaxDev] = {};
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (done[dev]) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    done[dev] = true;
+}
+} // namespace
+
 extern "C" int kcore_decompose_host(const int64_t *rowptr_h, const int32_t *colidx_h, int64_t n,
                                     int64_t m, int32_t *core_h, void *stream_,
                                     const kcore_options *opt, kcore_stats *stats)
@@ -369,6 +391,7 @@ extern "C" int kcore_decompose_host(const int64_t *rowptr_h, const int32_t *coli
     cudaStream_t st = (cudaStream_t)stream_;
     int64_t *d_rp = nullptr;
     int32_t *d_ci = nullptr, *d_core = nullptr;
+    keep_pool_warm();
     KC_CUDA(cudaMallocAsync((void **)&d_rp, sizeof(int64_t) * (size_t)(n + 1), st));
     KC_CUDA(cudaMallocAsync((void **)&d_ci, sizeof(int32_t) * (size_t)(m > 0 ? m : 1), st));
     KC_CUDA(cudaMallocAsync((void **)&d_core, sizeof(int32_t) * (size_t)n, st));
