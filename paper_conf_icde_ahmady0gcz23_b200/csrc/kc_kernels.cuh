@@ -57,10 +57,10 @@ constexpr int kWarps = kBlock / 32;
 #endif
 constexpr int kScanItems = KC_SCAN_ITEMS;        // alive-list entries per lane per warp step
 constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)
-// CTA-local routing budgets (arcs), chosen per level from the size of the
-// previous level: light levels keep their BFS local, heavy ones go grid-wide.
-constexpr int kLightLevelArcs = 4 << 20;
-constexpr int kHubLight = 32768, kSubLight = 32768, kPhaseLight = 262144;
+// CTA-local routing budgets (arcs): a claimed vertex with more arcs than
+// kHub, or one that would push the next local sub-round past kSub or the
+// CTA's phase total past kPhase, goes to the global queue (HUB phase) instead
+// of the CTA's own frontier (tuned on B200: DESIGN.md §8).
 #ifndef KC_HUB
 #define KC_HUB 32768
 #endif
@@ -70,7 +70,7 @@ constexpr int kHubLight = 32768, kSubLight = 32768, kPhaseLight = 262144;
 #ifndef KC_PHASE
 #define KC_PHASE 65536
 #endif
-constexpr int kHubHeavy = KC_HUB, kSubHeavy = KC_SUB, kPhaseHeavy = KC_PHASE;
+constexpr int kHub = KC_HUB, kSub = KC_SUB, kPhase = KC_PHASE;
 #ifndef KC_GSTAGE
 #define KC_GSTAGE 64
 #endif
@@ -131,7 +131,7 @@ struct Ctrl {
     int32_t phase, solo, k, level_min;
     int32_t compact, src_sel, dst_sel, alive_sel;
     int32_t src_single, alive_single;  // 1: the list is one contiguous run in segment 0
-    int32_t light;                     // budgets of this level (see kLightLevelArcs)
+    int32_t pad0;
     int32_t pad1;
     int64_t arcs_lvl0;                 // arcs walked when the level began
     int64_t pad2;
@@ -207,7 +207,7 @@ struct Smem {
     int32_t larc[2];
     int32_t lphase;      // local arcs accepted this phase
     int32_t removed;     // vertices removed by this CTA this phase (order not recorded)
-    int32_t fit;         // unused
+    int32_t pad_fit;
     int32_t kcur;        // scan: compaction cursor within the current segment
     int32_t seg_cache[2];     // length of this CTA's own segment in alive[x], as it last wrote it
     int32_t seg_cache_ok[2];  // (persistent kernel only; a k_phase launch starts without it)
@@ -921,7 +921,7 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
 
 // ------------------------------------------------------------------ LEVEL
 // Scan entries [lo,hi) of list `src` (nullptr: the identity, ids lo..hi-1)
-// with every warp of this CTA (Alg. 2): eight entries per lane in flight;
+// with every warp of this CTA (Alg. 2): kScanItems entries per lane in flight;
 // deg == k -> claim + route (local frontier or global queue); deg > k ->
 // min for the level skip and, when compacting, ballot compaction (Fig. 8(c))
 // into dst[0..) with a shared-memory cursor.  No block sync, no global atomics.
@@ -1060,10 +1060,10 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     if (threadIdx.x == 0) PROBE(30, c.k * 4 + c.phase);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
-        sm.lphase = 0; sm.removed = 0; sm.fit = 0;
-        sm.bud_hub = c.light ? kHubLight : kHubHeavy;
-        sm.bud_sub = c.light ? kSubLight : kSubHeavy;
-        sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
+        sm.lphase = 0; sm.removed = 0;
+        sm.bud_hub = kHub;
+        sm.bud_sub = kSub;
+        sm.bud_phase = kPhase;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
@@ -1102,10 +1102,10 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     if (threadIdx.x == 0) PROBE(30, c.k * 4 + c.phase);
     if (threadIdx.x == 0) {
         sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
-        sm.lphase = 0; sm.removed = 0; sm.fit = 0;
-        sm.bud_hub = c.light ? kHubLight : kHubHeavy;
-        sm.bud_sub = c.light ? kSubLight : kSubHeavy;
-        sm.bud_phase = c.light ? kPhaseLight : kPhaseHeavy;
+        sm.lphase = 0; sm.removed = 0;
+        sm.bud_hub = kHub;
+        sm.bud_sub = kSub;
+        sm.bud_phase = kPhase;
     }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
@@ -1180,8 +1180,6 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         }
         // level end
         if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
-        c.light = 0;  // adaptive budgets disabled: misjudge level jumps
-        (void)kLightLevelArcs;
         if (removed >= p.n) {
             c.phase = PH_DONE;
             c.solo = 0;
@@ -1315,7 +1313,6 @@ __device__ __forceinline__ void init_ctrl(Ctrl &z)
     z.level_min = INT_MAX;
     z.alive_sel = -1;
     z.src_sel = -1;
-    z.light = 0;
 }
 
 __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant__ KArgs A)
