@@ -91,3 +91,23 @@ def test_mpm_fixpoint_configs(name):
     ref = oracle.bz_core(r.cpu().numpy(), c.cpu().numpy())
     a, it = kc.kcore_mpm(r, c)
     assert np.array_equal(a.cpu().numpy(), ref), (name, it)
+
+
+@pytest.mark.slow
+def test_outputs_full_size_C2():
+    """Outputs at a BASELINE config's full size (C2: 4.2M vertices, 134M arcs)
+    against the oracle's deletion-definition k-core and induced subgraph."""
+    r, c = kcgen.generate_device(kcgen.CONFIGS["C2"])
+    rp, ci = r.cpu().numpy(), c.cpu().numpy()
+    core = kc.kcore_decompose(r, c)
+    kmax = int(core.max())
+    for k in (kmax // 2, kmax):
+        want = oracle.kcore_members(rp, ci, k)
+        mask, cnt = kc.kcore_kcore_mask(core, k)
+        assert np.array_equal(mask.cpu().numpy(), want) and cnt == int(want.sum()), k
+        shell = kc.kcore_kshell(core, k).cpu().numpy()
+        assert np.array_equal(shell, np.nonzero((core == k).cpu().numpy())[0]), k
+        srp, sci, vm = kc.kcore_kcore_subgraph(r, c, core, k)
+        orp, oci, ovm = oracle.induced_csr(rp, ci, want)
+        assert np.array_equal(srp.cpu().numpy(), orp) and np.array_equal(vm.cpu().numpy(), ovm), k
+        assert np.array_equal(sci.cpu().numpy(), oci), k
