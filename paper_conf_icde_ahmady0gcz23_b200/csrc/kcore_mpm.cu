@@ -148,6 +148,53 @@ __device__ __forceinline__ void small_vertex(const MArgs &A, int32_t v, int64_t 
     warp_append(ch && lane == 0, v, A.chg, &A.S->chg_len[t & 1]);
 }
 
+// h = max{h <= min(c, d) : N(h) >= h} over the capped estimates x[] (R
+// registers per lane) by a ballot-count binary search; also N(h).
+template <int R>
+__device__ __forceinline__ void hsearch(const int32_t (&x)[R], int32_t c, int64_t d, int &lo, int &nlo)
+{
+    int hi = (int)min((int64_t)c, d);
+    lo = 0;
+    nlo = (int)d;
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        int cnt = 0;
+#pragma unroll
+        for (int r = 0; r < R; r++) cnt += __popc(__ballot_sync(kFull, x[r] >= mid));
+        if (cnt >= mid) { lo = mid; nlo = cnt; } else hi = mid - 1;
+    }
+}
+
+// A1 for two vertices of <= 64 arcs at once: both gathers in flight together
+// (the small path is bound by the latency of the estimate gathers).
+__device__ __forceinline__ void small_pair(const MArgs &A, int32_t v0, int64_t b0, int64_t d0, int32_t v1,
+                                           int64_t b1, int64_t d1, int t)
+{
+    const int lane = threadIdx.x & 31;
+    const int32_t c0 = __ldcg(A.a + v0), c1 = __ldcg(A.a + v1);
+    int32_t x0[2], x1[2];
+#pragma unroll
+    for (int r = 0; r < 2; r++) {
+        const int64_t i = r * 32 + lane;
+        x0[r] = i < d0 ? __ldcg(A.a + __ldg(A.colidx + b0 + i)) : -1;
+        x1[r] = i < d1 ? __ldcg(A.a + __ldg(A.colidx + b1 + i)) : -1;
+    }
+#pragma unroll
+    for (int r = 0; r < 2; r++) { x0[r] = min(x0[r], c0); x1[r] = min(x1[r], c1); }
+    int h0, n0, h1, n1;
+    hsearch(x0, c0, d0, h0, n0);
+    hsearch(x1, c1, d1, h1, n1);
+    const bool ch0 = h0 != c0, ch1 = h1 != c1;
+    if (lane == 0) {
+        A.cnt[v0] = n0;
+        if (ch0) { A.a_new[v0] = h0; A.cstamp[v0] = t; }
+        A.cnt[v1] = n1;
+        if (ch1) { A.a_new[v1] = h1; A.cstamp[v1] = t; }
+    }
+    warp_append(ch0 && lane == 0, v0, A.chg, &A.S->chg_len[t & 1]);
+    warp_append(ch1 && lane == 0, v1, A.chg, &A.S->chg_len[t & 1]);
+}
+
 // A2: the whole CTA, vertex v with d > kSmall arcs
 __device__ void big_vertex(const MArgs &A, MSmem &sm, int32_t v, int t)  // t: iteration
 {
@@ -278,15 +325,25 @@ __global__ void __launch_bounds__(kB, 1) k_mpm(const __grid_constant__ MArgs A)
         const int64_t len = (t == 1) ? A.n : (int64_t)__ldcg(&S->act_len[t & 1]);
         const int32_t *act = A.act[t & 1];
         // A1: small vertices by warps, big ones deferred
-        for (int64_t i = gw; i < len; i += nw) {
-            const int32_t v = (t == 1) ? (int32_t)i : __ldcg(act + i);
-            const int64_t b = __ldg(A.rowptr + v), d = __ldg(A.rowptr + v + 1) - b;
-            if (d > kSmall) {
-                if (lane == 0) A.big[atomicAdd(&S->big_len[t & 1], 1ULL)] = v;
-            } else if (d > 0) {
-                small_vertex(A, v, b, d, t);
+        for (int64_t i = gw; i < len; i += 2 * nw) {  // entries i and i + nw
+            const int64_t j = i + nw;
+            const int32_t v0 = (t == 1) ? (int32_t)i : __ldcg(act + i);
+            const int32_t v1 = j < len ? ((t == 1) ? (int32_t)j : __ldcg(act + j)) : -1;
+            const int64_t b0 = __ldg(A.rowptr + v0), d0 = __ldg(A.rowptr + v0 + 1) - b0;
+            int64_t b1 = 0, d1 = 0;
+            if (v1 >= 0) { b1 = __ldg(A.rowptr + v1); d1 = __ldg(A.rowptr + v1 + 1) - b1; }
+            if (lane == 0) {
+                if (d0 > kSmall) A.big[atomicAdd(&S->big_len[t & 1], 1ULL)] = v0;
+                if (d1 > kSmall) A.big[atomicAdd(&S->big_len[t & 1], 1ULL)] = v1;
             }
-            if (lane == 0) { processed++; arcs += d; }
+            const bool s0 = d0 > 0 && d0 <= kSmall, s1 = v1 >= 0 && d1 > 0 && d1 <= kSmall;
+            if (s0 && s1 && d0 <= 64 && d1 <= 64) {
+                small_pair(A, v0, b0, d0, v1, b1, d1, t);
+            } else {
+                if (s0) small_vertex(A, v0, b0, d0, t);
+                if (s1) small_vertex(A, v1, b1, d1, t);
+            }
+            if (lane == 0) { processed += 1 + (v1 >= 0); arcs += d0 + d1; }
         }
         grid.sync();
         // A2: big vertices by whole CTAs
