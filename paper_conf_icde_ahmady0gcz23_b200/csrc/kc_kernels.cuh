@@ -57,6 +57,8 @@ constexpr int kWarps = kBlock / 32;
 #endif
 constexpr int kScanItems = KC_SCAN_ITEMS;        // alive-list entries per lane per warp step
 constexpr int kLCap = kBlock;        // local frontier capacity (entries; one per thread in the prefix scan)
+constexpr int kQCap = 1024;          // async drain: chunk queue capacity (chunks of <= 128 arcs)
+constexpr int kAsyncNx = 2;          // route target "async chunk queue" (lists 0/1 are the sub-round lists)
 // CTA-local routing budgets (arcs): a claimed vertex with more arcs than
 // kHub, or one that would push the next local sub-round past kSub or the
 // CTA's phase total past kPhase, goes to the global queue (HUB phase) instead
@@ -75,7 +77,10 @@ constexpr int kHub = KC_HUB, kSub = KC_SUB, kPhase = KC_PHASE;
 #define KC_GSTAGE 64
 #endif
 constexpr int kGStage = KC_GSTAGE;          // per-warp global-queue stage (any size; flushed 32 at a time)
-constexpr int kBloomBits = 1 << 20;  // 128 KB
+#ifndef KC_BLOOM_LOG2
+#define KC_BLOOM_LOG2 19
+#endif
+constexpr int kBloomBits = 1 << KC_BLOOM_LOG2;  // 64 KB: shared memory is taken from L1 (2^20 bits: C4 +5 %)
 constexpr int kBloomWords = kBloomBits / 32;
 #ifndef KC_BLOOM_MAXA
 #define KC_BLOOM_MAXA (1 << 18)
@@ -112,6 +117,9 @@ constexpr int kTraceFields = 8;
 #endif
 #ifndef KC_COMPACT_D
 #define KC_COMPACT_D 32 // compact the alive list once >= 1/KC_COMPACT_D of it is dead
+#endif
+#ifndef KC_ASYNC
+#define KC_ASYNC 0  // 1: CTA-local drain as an asynchronous chunk queue (no sub-round barriers)
 #endif
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
@@ -199,10 +207,19 @@ struct KArgs {
 };
 
 struct Smem {
-    int32_t lv[2][kLCap];
-    int32_t ld[2][kLCap];
-    int64_t lb[2][kLCap];
-    int64_t lpre[kLCap + 1];
+    union {
+        struct {  // sub-round lists (synchronous drain)
+            int32_t lv[2][kLCap];
+            int32_t ld[2][kLCap];
+            int64_t lb[2][kLCap];
+            int64_t lpre[kLCap + 1];
+        };
+        struct {  // chunk queue (asynchronous drain, KC_ASYNC)
+            int64_t qbeg[kQCap];  // chunk = colidx [qbeg, qbeg + qlen)
+            int32_t qlen[kQCap];
+            int32_t qflag[kQCap];  // == qepoch once the chunk is written
+        };
+    };
     int32_t lcnt[2];
     int32_t larc[2];
     int32_t lphase;      // local arcs accepted this phase
@@ -224,6 +241,8 @@ struct Smem {
     int32_t bloom_on;
     Ctrl ctrl;
     Snap snap;
+    int32_t qhead, qtail, qpend, qepoch;
+    unsigned long long qwalked;
     uint32_t bloom[kBloomWords];
 };
 
@@ -279,8 +298,8 @@ __device__ __forceinline__ void probe(int tag, int64_t val)
 #define PROBE(tag, val) ((void)0)
 #endif
 
-__device__ __forceinline__ uint32_t bloom_h1(uint32_t v) { return (v * 0x9E3779B1u) >> 12; }
-__device__ __forceinline__ uint32_t bloom_h2(uint32_t v) { return ((v ^ (v >> 15)) * 0x85EBCA6Bu) >> 12; }
+__device__ __forceinline__ uint32_t bloom_h1(uint32_t v) { return (v * 0x9E3779B1u) >> (32 - KC_BLOOM_LOG2); }
+__device__ __forceinline__ uint32_t bloom_h2(uint32_t v) { return ((v ^ (v >> 15)) * 0x85EBCA6Bu) >> (32 - KC_BLOOM_LOG2); }
 
 __device__ __forceinline__ bool bloom_maybe(const Smem &sm, uint32_t v)
 {
@@ -542,7 +561,53 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
     }
     unsigned lm = 0;  // candidates that go to the local list
     int lbase = 0;
-    if (ctot) {
+    if (KC_ASYNC && nx == kAsyncNx && ctot) {
+        // chunks of <= 128 arcs per candidate into the CTA's async queue
+        int nc[4], mine = 0;
+#pragma unroll
+        for (int r = 0; r < 4; r++) {
+            nc[r] = ((cm >> r) & 1u) ? (dd[r] + kBatch - 1) / kBatch : 0;
+            mine += nc[r];
+        }
+        int incl = mine;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int t = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl += t;
+        }
+        const int tot = __shfl_sync(kFull, incl, 31);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sumd += __shfl_xor_sync(kFull, sumd, o);
+        int ok = 0, base = 0;
+        if (lane == 0) {
+            const int op = atomicAdd(&sm.lphase, sumd);
+            if (op + sumd <= sm.bud_phase) {
+                int t = *(volatile int *)&sm.qtail;
+                while (t + tot <= kQCap) {
+                    const int o2 = atomicCAS(&sm.qtail, t, t + tot);
+                    if (o2 == t) { ok = 1; base = t; break; }
+                    t = o2;
+                }
+                if (ok) atomicAdd(&sm.qpend, tot);  // before any chunk is visible
+            }
+        }
+        ok = __shfl_sync(kFull, ok, 0);
+        base = __shfl_sync(kFull, base, 0);
+        if (ok) {
+            int pos = base + incl - mine;
+            const int ep = sm.qepoch;
+#pragma unroll
+            for (int r = 0; r < 4; r++) {
+                for (int q = 0; q < nc[r]; q++, pos++) {
+                    sm.qbeg[pos] = bb[r] + (int64_t)q * kBatch;
+                    sm.qlen[pos] = min(kBatch, dd[r] - q * kBatch);
+                    __threadfence_block();
+                    *(volatile int32_t *)&sm.qflag[pos] = ep;
+                }
+            }
+            lm = cm;
+        }
+    } else if (ctot) {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) sumd += __shfl_xor_sync(kFull, sumd, o);
         int ok = 0;
@@ -827,6 +892,68 @@ __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, b
     return walked;
 }
 
+// Asynchronous CTA-local drain (KC_ASYNC; the PKC idea of P:L63 -- no
+// sub-level synchronisation -- at CTA scope): the frontier lives in a
+// shared-memory queue of chunks (<= 128 arcs of one row); each warp pops a
+// chunk, walks it, and pushes the chunks of the vertices it claimed.
+// qpend counts pushed-but-unfinished chunks; the drain ends when it is 0.
+__device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool use_bloom, bool atom_only,
+                                     int &lmin, int &gcnt)
+{
+    const int lane = threadIdx.x & 31;
+    const uint64_t pol = deg_policy();
+    const int ep = sm.qepoch;
+    int64_t walked = 0;
+    while (true) {
+        int idx = 0;
+        if (lane == 0) {
+            idx = atomicAdd(&sm.qhead, 1);
+            if (idx >= kQCap) {
+                idx = -1;
+            } else {
+                while (*(volatile int32_t *)&sm.qflag[idx] != ep) {
+                    if (*(volatile int32_t *)&sm.qpend == 0) { idx = -1; break; }
+                }
+            }
+        }
+        idx = __shfl_sync(kFull, idx, 0);
+        if (idx < 0) break;
+        __threadfence_block();
+        const int64_t beg = sm.qbeg[idx];
+        const int len = sm.qlen[idx];
+        int32_t u[kUnroll];
+#pragma unroll
+        for (int r = 0; r < kUnroll; r++) {
+            const int my = r * 32 + lane;
+            u[r] = my < len ? ld_stream_i32(A.colidx + beg + my) : -1;
+        }
+        if (use_bloom) {
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++)
+                if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
+        }
+        int old[kUnroll];
+#pragma unroll
+        for (int r = 0; r < kUnroll; r++) {
+            const int32_t d = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
+            old[r] = d > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
+        }
+        unsigned hm = 0;
+#pragma unroll
+        for (int r = 0; r < kUnroll; r++) {
+            if (old[r] == k + 1) hm |= 1u << r;
+            else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
+        }
+        if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, k, kAsyncNx, u[0], u[1], u[2], u[3], hm, gcnt);
+        walked += len;
+        __syncwarp();
+        if (lane == 0) atomicSub(&sm.qpend, 1);
+    }
+    if (lane == 0 && walked) atomicAdd(&sm.qwalked, (unsigned long long)walked);
+    __syncthreads();
+    return (int64_t)sm.qwalked;
+}
+
 // Bloom filter of the alive list at level start (built once per level).
 __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
 {
@@ -883,7 +1010,8 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
     const int lane = threadIdx.x & 31;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (threadIdx.x == 0) sm.removed = 0;
+    if (threadIdx.x == 0) { sm.removed = 0; sm.qepoch = 0; }
+    for (int i = threadIdx.x; i < kQCap; i += kBlock) sm.qflag[i] = -1;
     __syncthreads();
     // The 0-shell is the isolated vertices: nothing can reach them, so
     // they are removed here -- claim bit set, core 0, counted as removed -- and
@@ -1000,7 +1128,7 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
                 if (du[j] > 0) prefetch_row(A.colidx, b0[j], b0[j] + du[j]);
             if constexpr (KC_ROUTE4 && kScanItems == 4) {
                 route_won4(A, sm, wib, wm, vv[0], vv[1], vv[2], vv[3], du[0], du[1], du[2], du[3], b0[0], b0[1],
-                           b0[2], b0[3], 0, gcnt);
+                           b0[2], b0[3], KC_ASYNC ? kAsyncNx : 0, gcnt);
             } else {
 #pragma unroll
                 for (int j = 0; j < kScanItems; j++) route_won(A, sm, wib, (wm >> j) & 1u, vv[j], du[j], b0[j], 0, gcnt);
@@ -1064,6 +1192,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.bud_hub = kHub;
         sm.bud_sub = kSub;
         sm.bud_phase = kPhase;
+        sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qepoch++; sm.qwalked = 0ULL;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
@@ -1072,7 +1201,8 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_LOCAL;
     int64_t subs = 0, tmax = 0;
-    const int64_t walked = local_drain(A, sm, c.k, 0, bl, ao, lmin, gcnt, &subs, &tmax);
+    const int64_t walked = KC_ASYNC ? local_drain_async(A, sm, c.k, bl, ao, lmin, gcnt)
+                                    : local_drain(A, sm, c.k, 0, bl, ao, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
@@ -1106,6 +1236,7 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
         sm.bud_hub = kHub;
         sm.bud_sub = kSub;
         sm.bud_phase = kPhase;
+        sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qepoch++; sm.qwalked = 0ULL;
     }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
@@ -1113,12 +1244,14 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_HUB;
     const int64_t a0 = c.as + gw * C;
     if (a0 < c.ae)
-        walk<false>(A, sm, c.k, 0, 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt, KC_CF_HUB);
+        walk<false>(A, sm, c.k, 0, KC_ASYNC ? kAsyncNx : 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt,
+                    KC_CF_HUB);
     int64_t walked = cta_arcs;
     __syncthreads();
     cta_time(A, c, 1);
     int64_t subs = 0, tmax = 0;
-    walked += local_drain(A, sm, c.k, 0, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
+    walked += KC_ASYNC ? local_drain_async(A, sm, c.k, bl, ao && KC_AO_LOCAL, lmin, gcnt)
+                       : local_drain(A, sm, c.k, 0, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
@@ -1374,7 +1507,9 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(const __grid_constant__ KAr
         sm.bloom_on = 0;
         sm.bloom_level = -1;
         sm.seg_cache_ok[0] = sm.seg_cache_ok[1] = 0;
+        sm.qepoch = 0;
     }
+    for (int i = threadIdx.x; i < kQCap; i += kBlock) sm.qflag[i] = -1;
     __syncthreads();
     const Ctrl &c = sm.ctrl;
     if (c.phase == PH_INIT) phase_init(A, sm);
