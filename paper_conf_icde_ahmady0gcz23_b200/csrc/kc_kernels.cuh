@@ -119,7 +119,11 @@ constexpr int kTraceFields = 8;
 #define KC_COMPACT_D 32 // compact the alive list once >= 1/KC_COMPACT_D of it is dead
 #endif
 #ifndef KC_ASYNC
-#define KC_ASYNC 0  // 1: CTA-local drain as an asynchronous chunk queue (no sub-round barriers)
+#define KC_ASYNC 2  // 1: CTA-local drain as an asynchronous chunk queue (no sub-round barriers);
+                    // 2: per CTA and phase, async when the frontier's rows are long
+#endif
+#ifndef KC_ASYNC_MINAVG
+#define KC_ASYNC_MINAVG 64  // KC_ASYNC 2: async when the local frontier averages >= this many arcs per vertex
 #endif
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
@@ -954,6 +958,41 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
     return (int64_t)sm.qwalked;
 }
 
+// The CTA's drain of its local frontier (list 0 or, KC_ASYNC 1, the chunk
+// queue).  KC_ASYNC 2 picks per CTA and phase: long rows (a chain of hubs-to-
+// be) drain asynchronously, many short rows keep the packed sub-rounds.
+__device__ int64_t drain(const KArgs &A, Smem &sm, const int k, bool use_bloom, bool atom_only, int &lmin,
+                         int &gcnt, int64_t *subs, int64_t *tmax)
+{
+    if (KC_ASYNC == 1) return local_drain_async(A, sm, k, use_bloom, atom_only, lmin, gcnt);
+    if (KC_ASYNC == 2) {
+        __syncthreads();
+        const int L = min(sm.lcnt[0], kLCap);
+        int32_t v = 0, d = 0;
+        int64_t b = 0;
+        if ((int)threadIdx.x < L) { v = sm.lv[0][threadIdx.x]; d = sm.ld[0][threadIdx.x]; b = sm.lb[0][threadIdx.x]; }
+        const int nc = (int)threadIdx.x < L ? (d + kBatch - 1) / kBatch : 0;
+        unsigned long long tq, tr;
+        block_excl_scan2(sm, (unsigned long long)nc, (unsigned long long)d, tq, tr);
+        const int64_t chunks = (int64_t)sm.tot_q, arcs = (int64_t)sm.tot_q2;
+        if (L > 0 && arcs >= (int64_t)KC_ASYNC_MINAVG * L && chunks <= kQCap) {
+            __syncthreads();  // everyone holds its list entry: the queue may overwrite the lists
+            const int ep = sm.qepoch;
+            for (int q = 0; q < nc; q++) {
+                const int pos = (int)tq + q;
+                sm.qbeg[pos] = b + (int64_t)q * kBatch;
+                sm.qlen[pos] = min(kBatch, d - q * kBatch);
+                sm.qflag[pos] = ep;
+            }
+            (void)v;
+            if (threadIdx.x == 0) { sm.qtail = (int)chunks; sm.qpend = (int)chunks; sm.qhead = 0; }
+            __syncthreads();
+            return local_drain_async(A, sm, k, use_bloom, atom_only, lmin, gcnt);
+        }
+    }
+    return local_drain(A, sm, k, 0, use_bloom, atom_only, lmin, gcnt, subs, tmax);
+}
+
 // Bloom filter of the alive list at level start (built once per level).
 __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
 {
@@ -1128,7 +1167,7 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
                 if (du[j] > 0) prefetch_row(A.colidx, b0[j], b0[j] + du[j]);
             if constexpr (KC_ROUTE4 && kScanItems == 4) {
                 route_won4(A, sm, wib, wm, vv[0], vv[1], vv[2], vv[3], du[0], du[1], du[2], du[3], b0[0], b0[1],
-                           b0[2], b0[3], KC_ASYNC ? kAsyncNx : 0, gcnt);
+                           b0[2], b0[3], KC_ASYNC == 1 ? kAsyncNx : 0, gcnt);
             } else {
 #pragma unroll
                 for (int j = 0; j < kScanItems; j++) route_won(A, sm, wib, (wm >> j) & 1u, vv[j], du[j], b0[j], 0, gcnt);
@@ -1201,8 +1240,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_LOCAL;
     int64_t subs = 0, tmax = 0;
-    const int64_t walked = KC_ASYNC ? local_drain_async(A, sm, c.k, bl, ao, lmin, gcnt)
-                                    : local_drain(A, sm, c.k, 0, bl, ao, lmin, gcnt, &subs, &tmax);
+    const int64_t walked = drain(A, sm, c.k, bl, ao, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
@@ -1244,14 +1282,13 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_HUB;
     const int64_t a0 = c.as + gw * C;
     if (a0 < c.ae)
-        walk<false>(A, sm, c.k, 0, KC_ASYNC ? kAsyncNx : 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt,
+        walk<false>(A, sm, c.k, 0, KC_ASYNC == 1 ? kAsyncNx : 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt,
                     KC_CF_HUB);
     int64_t walked = cta_arcs;
     __syncthreads();
     cta_time(A, c, 1);
     int64_t subs = 0, tmax = 0;
-    walked += KC_ASYNC ? local_drain_async(A, sm, c.k, bl, ao && KC_AO_LOCAL, lmin, gcnt)
-                       : local_drain(A, sm, c.k, 0, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
+    walked += drain(A, sm, c.k, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
     cta_time(A, c, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
