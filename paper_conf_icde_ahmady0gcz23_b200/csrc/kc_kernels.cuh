@@ -128,6 +128,9 @@ constexpr int kTraceFields = 8;
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
 #endif
+#ifndef KC_TAGBAR
+#define KC_TAGBAR 0  // 1: grid barrier publishes the snapshot as generation-tagged words (no release flag)
+#endif
 #ifndef KC_AO_HUB
 #define KC_AO_HUB 1
 #endif
@@ -183,6 +186,7 @@ struct State {
     alignas(128) uint32_t bar_count;            // grid barrier arrivals (monotone)
     alignas(128) uint32_t bar_gen;              // grid barrier generation
     Snap snap[2];                               // counters at barrier gen, by gen & 1
+    alignas(128) unsigned long long tsnap[8];   // KC_TAGBAR: (gen & 0xffff) << 48 | value, see grid_barrier
     alignas(128) unsigned long long arcs_walked;
     alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
     alignas(128) Params prm;
@@ -1412,6 +1416,18 @@ __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &s
 }
 
 // Grid barrier; the last arriver snapshots+resets the counters.
+//
+// KC_TAGBAR: the last arriver publishes the snapshot as six 64-bit words, each
+// tagged with the new generation in its top 16 bits, after a release fence;
+// the others poll all six words at once (independent relaxed loads, one round
+// trip per poll) until every tag is the new generation, then fence (acquire).
+// No separate flag store/poll and no second read of the snapshot after the
+// flag: one memory round trip less on both sides of every barrier.  A waiter
+// of generation g finishes reading before it arrives at barrier g+1, so one
+// set of words suffices; a stale word carries tag g != g+1 (mod 2^16).
+constexpr int kTagShift = 48;
+constexpr unsigned long long kTagVal = (1ULL << kTagShift) - 1ULL;
+
 __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
 {
     __syncthreads();
@@ -1427,6 +1443,41 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
         const uint32_t gen = t / (uint32_t)gridDim.x;
         PROBE(35, t);
         Snap sn;
+#if KC_TAGBAR
+        const unsigned long long tag = (unsigned long long)((gen + 1u) & 0xffffu) << kTagShift;
+        if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
+            sn = take_snapshot(S, gridDim.x);
+            fence_acq_rel_gpu();  // release: everything this CTA observed before the words
+            st_relaxed_u64(&S->tsnap[0], tag | sn.ord);
+            st_relaxed_u64(&S->tsnap[1], tag | sn.alive_out);
+            st_relaxed_u64(&S->tsnap[2], tag | (unsigned long long)(uint32_t)sn.min);
+            st_relaxed_u64(&S->tsnap[3], tag | (sn.gq >> kArcBits));
+            st_relaxed_u64(&S->tsnap[4], tag | (sn.gq & kArcMask));
+            st_relaxed_u64(&S->tsnap[5], tag | sn.arcs);
+        } else {
+            unsigned long long w0, w1, w2, w3, w4, w5;
+            while (true) {
+                w0 = ld_relaxed_u64(&S->tsnap[0]);
+                w1 = ld_relaxed_u64(&S->tsnap[1]);
+                w2 = ld_relaxed_u64(&S->tsnap[2]);
+                w3 = ld_relaxed_u64(&S->tsnap[3]);
+                w4 = ld_relaxed_u64(&S->tsnap[4]);
+                w5 = ld_relaxed_u64(&S->tsnap[5]);
+                const unsigned long long hi = ~kTagVal;
+                if (((w0 & hi) == tag) & ((w1 & hi) == tag) & ((w2 & hi) == tag) & ((w3 & hi) == tag) &
+                    ((w4 & hi) == tag) & ((w5 & hi) == tag))
+                    break;
+            }
+            fence_acq_rel_gpu();  // acquire: pairs with the last arriver's fence
+            PROBE(34, 0);
+            sn.ord = w0 & kTagVal;
+            sn.alive_out = w1 & kTagVal;
+            sn.min = (int32_t)(uint32_t)(w2 & 0xffffffffULL);
+            sn.gq = ((w3 & kTagVal) << kArcBits) | (w4 & kTagVal);
+            sn.arcs = w5 & kTagVal;
+            sn.pad = 0;
+        }
+#else
         if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
             sn = take_snapshot(S, gridDim.x);
             S->snap[(gen + 1u) & 1u] = sn;
@@ -1443,6 +1494,7 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
             sn.min = ld_relaxed_i32(&ps->min);
             sn.pad = 0;
         }
+#endif
         sm.snap = sn;
     }
     __syncthreads();
@@ -1584,6 +1636,7 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
         S->min_next = INT_MAX;
         S->bar_count = 0u;
         S->bar_gen = 0u;
+        for (int i = 0; i < 8; i++) S->tsnap[i] = 0ULL;  // tag 0: generation 0 is never awaited
         S->arcs_walked = 0ULL;
         Ctrl z;
         init_ctrl(z);
