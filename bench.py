@@ -144,6 +144,68 @@ def run_reference(args):
     return 0
 
 
+def _lib_sha():
+    import hashlib
+    try:
+        import paper_conf_icde_ahmady0gcz23_b200 as kc
+        with open(kc.LIB_PATH, "rb") as f:
+            return hashlib.sha256(f.read()).hexdigest()
+    except Exception:
+        return None
+
+
+def _cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return None
+
+
+def per_config(args, kc, kcgen, flush, stream, peak, with_oracle=True):
+    """C1-C3 (BASELINE.json configs[0..2]): kernel time median/min/std over
+    K steps (L2 flushed between steps), roofline fraction with the same B_min
+    formula, bit-exact parity against the oracle (test infrastructure, the
+    cpu_baseline leg)."""
+    import torch
+    out = {}
+    for name, desc in (("C1", "rmat-s16-ef16"), ("C2", "er-4M-d32"), ("C3", "chunglu-4M-70M-g2.1")):
+        spec = kcgen.CONFIGS[name]
+        rp, ci = kcgen.generate_device(spec)
+        n, m = rp.numel() - 1, ci.numel()
+        ws = torch.empty(kc.kcore_workspace_size(n, m), dtype=torch.uint8, device=rp.device)
+        core = torch.empty(n, dtype=torch.int32, device=rp.device)
+        for _ in range(args.warmup):
+            kc.kcore_decompose(rp, ci, core_out=core, workspace=ws)
+        ks = []
+        st = None
+        for _ in range(args.steps):
+            flush.fill_(1)
+            _, st = kc.kcore_decompose(rp, ci, core_out=core, workspace=ws, stats=True)
+            ks.append(st.kernel_ms)
+        med = statistics.median(ks)
+        b_min = 4 * m + 8 * (n + 1) + 8 * n + 4 * n + 4 * st.scanned + 8 * n
+        d = {"workload": desc, "n": n, "arcs": m, "m_undirected": m // 2,
+             "kernel_ms_median": med, "kernel_ms_min": min(ks),
+             "kernel_ms_std": statistics.pstdev(ks) if len(ks) > 1 else 0.0,
+             "medges_per_s": m / 2 / (med * 1e-3) / 1e6,
+             "roofline_frac": b_min / (med * 1e-3) / 1e9 / peak, "algorithmic_bytes": b_min,
+             "levels": st.levels, "phases": st.phases, "kmax": st.kmax}
+        if with_oracle:
+            import oracle
+            rp_h, ci_h = rp.cpu().numpy(), ci.cpu().numpy()
+            t0 = time.perf_counter()
+            ref = oracle.bz_core(rp_h, ci_h)
+            d["oracle_s"] = time.perf_counter() - t0
+            d["parity"] = bool((ref == core.cpu().numpy()).all())
+        out[name] = d
+        del rp, ci, ws, core
+        torch.cuda.empty_cache()
+    return out
+
+
 def run_gpu(args):
     import torch
     world, rank, local, dist = _dist()
@@ -252,11 +314,20 @@ def run_gpu(args):
     scanned = statistics.mean(s.scanned for s in stats)
     b_min = 4 * m_arcs + 8 * (n + 1) + 8 * n + 4 * n + 4 * scanned + 8 * n  # SURVEY 8(d) B_min
     achieved = b_min / (kern_ms * 1e-3) / 1e9
-    traffic = None
+    # DRAM traffic of the dominant kernel: from the committed `ncu --set full`
+    # capture ONLY if that capture profiled this very library binary (sha256
+    # recorded in the capture); otherwise null.  (ncu cannot run inside the
+    # timed bench; profiles/README.md has the capture command.)
+    traffic, traffic_src = None, None
+    lib_sha = _lib_sha()
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic_C4.json")
-    if os.path.exists(tpath):
+    if os.path.exists(tpath) and world == 1 and not args.force_mg:
         try:
-            traffic = json.load(open(tpath)).get("dram_bytes_per_launch")
+            tj = json.load(open(tpath))
+            if tj.get("lib_sha256") == lib_sha:
+                traffic = tj.get("dram_bytes_per_launch")
+                traffic_src = {"file": "profiles/ncu_traffic_C4.json", "lib_sha256": lib_sha,
+                               "window_off_bytes": tj.get("dram_bytes_per_launch_window_off")}
         except Exception:
             traffic = None
     line = {
@@ -268,8 +339,14 @@ def run_gpu(args):
                    "m_undirected": m_und, "arcs": m_arcs, "l2": "flushed between steps (512 MiB write); "
                    "colidx 4 GB > L2", "parallelism": f"vertex-range x{world}" if world > 1 else "1 GPU"},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                     "algorithmic_bytes": b_min, "kernel_ms": kern_ms},
+                     "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
+                     "peak_source": peak_src, "algorithmic_bytes": b_min, "kernel_ms": kern_ms},
+        "timing": {"step_ms_median": statistics.median(step_ms), "step_ms_min": min(step_ms),
+                   "step_ms_mean": statistics.mean(step_ms),
+                   "step_ms_std": statistics.pstdev(step_ms) if len(step_ms) > 1 else 0.0,
+                   "kernel_ms_median": statistics.median(s.kernel_ms for s in stats),
+                   "kernel_ms_min": min(s.kernel_ms for s in stats)},
+        "lib_sha256": lib_sha,
         "gpu_launches": int(sum(s.launches for s in stats)),  # counted by the library, timed steps only
         "e2e": e2e,
         "clocks": clk,
@@ -290,16 +367,29 @@ def run_gpu(args):
                            "ms_per_step": statistics.mean(mm), "iterations": it_m,
                            "arcs_gathered": st_m.arcs_walked, "equals_peel": bool(torch.equal(a_m, core))}
         del a_m
+    if world == 1 and not args.force_mg and not args.no_configs:
+        # the other single-GPU configs (BASELINE.json configs[0..2]) with the same protocol
+        line["per_config"] = per_config(args, kc, kcgen, flush, stream, peak,
+                                        with_oracle=not args.no_cpu_baseline)
     if world == 1 and not args.no_cpu_baseline and not args.force_mg:
         import oracle
         rp_h, ci_h = rowptr.cpu().numpy(), colidx.cpu().numpy()
-        t0 = time.perf_counter()
-        ref = oracle.bz_core(rp_h, ci_h)
-        dt = time.perf_counter() - t0
+        dts = []
+        for _ in range(3):  # the paper's CPU protocol: mean of 3 runs
+            t0 = time.perf_counter()
+            ref = oracle.bz_core(rp_h, ci_h)
+            dts.append(time.perf_counter() - t0)
+        dt = statistics.mean(dts)
         ok = bool((ref == core.cpu().numpy()).all())
+        # I2 + I4 certificate on the device's own peel order: exactness without the oracle
+        order = torch.empty(n, dtype=torch.int32, device=dev)
+        core2, _ = kc.kcore_decompose(rowptr, colidx, order_out=order, stats=True)
+        cert = oracle.check_certificate(rp_h, ci_h, core2.cpu().numpy(), order.cpu().numpy()) == 0
         line["cpu_baseline"] = {"value": m_und / dt / 1e6, "unit": "Medges/s", "cores": 1, "kind": "oracle",
-                                "sample": f"serial BZ on the full {WORKLOAD} graph, once ({dt:.1f} s); host "
-                                          f"has {os.cpu_count()} cores", "parity": ok}
+                                "sample": f"serial BZ on the full {WORKLOAD} graph, mean of 3 runs "
+                                          f"({', '.join(f'{x:.1f}' for x in dts)} s)",
+                                "host_cpu_model": _cpu_model(), "host_nproc": os.cpu_count(),
+                                "parity": ok, "certificate_ok": bool(cert)}
     print(json.dumps(line), flush=True)
     if dist.is_initialized():
         dist.destroy_process_group()
@@ -315,6 +405,7 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-mpm", action="store_true", help="skip the MPM context measurement")
     ap.add_argument("--force-mg", action="store_true", help="run the multi-GPU path even at N=1")
+    ap.add_argument("--no-configs", action="store_true", help="skip the C1-C3 per-config measurements")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

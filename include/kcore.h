@@ -72,6 +72,10 @@ typedef enum {
                                 /* raising cudaLimitPersistingL2CacheSize (device-wide,   */
                                 /* never lowered) to the window size if it is smaller, and */
                                 /* returns the lines to normal priority after the kernel. */
+#define KCORE_FLAG_NO_RED 4     /* ablation: heavy HUB phases keep returning atomicSub     */
+                                /* (default: phases walking >= 2^21 arcs over an alive set */
+                                /* <= 1/8 of them use non-returning red.global.add and a   */
+                                /* rescan of the alive list at the same k)      */
 
 /* Algorithms selectable through kcore_options.algo. */
 #define KCORE_ALGO_PERSISTENT 0 /* default: one persistent kernel, device-resident loop */

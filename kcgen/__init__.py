@@ -172,6 +172,39 @@ def generate_device(spec: GraphSpec, v_begin: int = 0, v_end: int | None = None,
         return rowptr, colidx[:m]
 
 
+def generate_device_chunked(spec: GraphSpec, chunks: int = 16, device=None):
+    """The whole graph's CSR on the device, generated in `chunks` owner ranges
+    (each range regenerates every edge and keeps the arcs whose source it
+    owns), written straight into one colidx buffer of capacity 2*num_edges.
+    For graphs whose one-shot sort buffers would not fit next to the CSR
+    (C5: 8.6 G candidate arcs).  Byte-identical to generate_device(spec)."""
+    import torch
+
+    device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
+    n = spec.num_vertices
+    p = spec._c()
+    lib = _load()
+    with torch.cuda.device(device):
+        stream = torch.cuda.current_stream(device).cuda_stream
+        cap = 2 * spec.num_edges
+        colidx = torch.empty(cap, dtype=torch.int32, device=device)
+        rowptr = torch.empty(n + 1, dtype=torch.int64, device=device)
+        rowptr[0] = 0
+        off = 0
+        bounds = [n * i // chunks for i in range(chunks + 1)]
+        for vb, ve in zip(bounds[:-1], bounds[1:]):
+            rp = torch.empty(ve - vb + 1, dtype=torch.int64, device=device)
+            m = lib.kcg_device_generate(ctypes.byref(p), vb, ve, rp.data_ptr(), colidx.data_ptr() + 4 * off,
+                                        cap - off, stream)
+            if m < 0:
+                raise RuntimeError(f"kcg_device_generate({vb},{ve}) failed: {m}")
+            rowptr[vb + 1:ve + 1] = rp[1:] + off
+            off += m
+            del rp
+        torch.cuda.synchronize(device)
+        return rowptr, colidx[:off]
+
+
 def csr_from_edges(n: int, edges):
     """CSR of a hand-written edge list: symmetrised, self-loops dropped,
     duplicates merged, rows sorted (reading R2)."""

@@ -39,6 +39,7 @@ ALGO_PERSISTENT = 0
 ALGO_HOSTLOOP = 1
 FLAG_NO_BLOOM = 1
 FLAG_NO_L2_PERSIST = 2
+FLAG_NO_RED = 4
 
 # every symbol include/kcore.h declares (checked by tests/test_abi.py)
 EXPORTS = (
@@ -179,7 +180,7 @@ def _check_csr_tensors(rowptr, colidx):
 def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=None,
                     algo: int = ALGO_PERSISTENT, blocks_per_sm: int = 0, solo_arcs: int = 0,
                     solo_scan: int = 0, bloom: bool = True, trace=None,
-                    trace_cta=None, stats: bool = False, l2_persist: bool = True):
+                    trace_cta=None, stats: bool = False, l2_persist: bool = True, red: bool = True):
     """Core numbers of the graph (rowptr int64[n+1], colidx int32[m] CUDA tensors).
 
     Runs on the current stream of the tensors' device.  Returns an int32 tensor
@@ -197,7 +198,8 @@ def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=
                    workspace.numel() * workspace.element_size() if workspace is not None else 0,
                    trace.data_ptr() if trace is not None else None,
                    trace.shape[0] if trace is not None else 0,
-                   (0 if bloom else FLAG_NO_BLOOM) | (0 if l2_persist else FLAG_NO_L2_PERSIST), 0,
+                   (0 if bloom else FLAG_NO_BLOOM) | (0 if l2_persist else FLAG_NO_L2_PERSIST) |
+                   (0 if red else FLAG_NO_RED), 0,
                    trace_cta.data_ptr() if trace_cta is not None else None)
     st = _Stats()
     with torch.cuda.device(dev):

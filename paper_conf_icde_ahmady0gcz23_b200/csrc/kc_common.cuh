@@ -171,4 +171,31 @@ __device__ __forceinline__ unsigned lanemask_lt()
     return m;
 }
 
+// Ballot scan of Fig. 8(c): every lane of the warp
+// contributes a 0/1 predicate; `bits` = __ballot_sync of them, the return value
+// = the lane's EXCLUSIVE prefix count (the number of set predicates in lower
+// lanes, Fig. 8's a[j]).  The warp's total is __popc(bits), by which one lane
+// advances the append cursor e (Fig. 8, Lines 3-5).
+__device__ __forceinline__ int ballot_excl(bool p, unsigned &bits)
+{
+    bits = __ballot_sync(0xffffffffu, p);
+    return __popc(bits & lanemask_lt());
+}
+
+// Warp-aggregated append (Fig. 8, Lines 1-8): lanes with p write v to
+// buf[e_old + a[j]]; the lowest active lane advances *e by the warp's count in
+// ONE atomicAdd and broadcasts e_old.  Returns the warp's count.
+__device__ __forceinline__ int warp_append(bool p, int32_t v, int32_t *buf, int *e)
+{
+    unsigned bits;
+    const int a = ballot_excl(p, bits);
+    if (bits == 0u) return 0;
+    const int lead = __ffs(bits) - 1;
+    int base = 0;
+    if ((int)(threadIdx.x & 31) == lead) base = atomicAdd(e, __popc(bits));
+    base = __shfl_sync(0xffffffffu, base, lead);
+    if (p) buf[base + a] = v;
+    return __popc(bits);
+}
+
 } // namespace kc

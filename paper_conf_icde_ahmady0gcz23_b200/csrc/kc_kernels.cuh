@@ -140,13 +140,26 @@ constexpr int kTraceFields = 8;
 #ifndef KC_AO_ALWAYS
 #define KC_AO_ALWAYS 1
 #endif
+// Heavy HUB phases with non-returning decrements (walk_red) followed by a
+// rescan of the alive list at the same k: used when the phase walks at least
+// KC_RED_MIN arcs and the alive set is at most 1/KC_RED_RATIO of them (the
+// rescan then costs far less than the returns it saves).  0 disables.
+#ifndef KC_RED_MIN
+#define KC_RED_MIN (1 << 21)
+#endif
+#ifndef KC_RED_RATIO
+#define KC_RED_RATIO 8
+#endif
+#ifndef KC_RED_UNROLL
+#define KC_RED_UNROLL 8
+#endif
 enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
 struct Ctrl {
     int32_t phase, solo, k, level_min;
     int32_t compact, src_sel, dst_sel, alive_sel;
     int32_t src_single, alive_single;  // 1: the list is one contiguous run in segment 0
-    int32_t pad0;
+    int32_t red;                       // HUB phase walks with non-returning decrements (then a rescan)
     int32_t pad1;
     int64_t arcs_lvl0;                 // arcs walked when the level began
     int64_t pad2;
@@ -175,7 +188,7 @@ struct Params {
     int32_t solo_arcs;  // HUB phases with <= this many arcs run solo
     int32_t solo_scan;  // LEVEL phases over <= this many entries run solo
     int32_t bloom;      // 0 disables the Bloom filter
-    int32_t pad;
+    int32_t red;        // 0 disables non-returning heavy HUB walks (KC_RED_MIN)
 };
 
 struct State {
@@ -222,12 +235,14 @@ struct Smem {
             int64_t lb[2][kLCap];
             int64_t lpre[kLCap + 1];
         };
-        struct {  // chunk queue (asynchronous drain, KC_ASYNC)
-            int64_t qbeg[kQCap];  // chunk = colidx [qbeg, qbeg + qlen)
-            int32_t qlen[kQCap];
-            int32_t qflag[kQCap];  // == qepoch once the chunk is written
-        };
     };
+    // Chunk queue of the asynchronous drain (KC_ASYNC): slot = one 64-bit word
+    // published and consumed with shared-memory atomics -- colidx begin in bits
+    // [0,34), chunk length - 1 in bits [34,41), bit 63 = valid; 0 = empty.  A
+    // popper takes the word with atomicExch(slot, 0), so every slot is empty
+    // again when the drain ends (qpend == 0 => every pushed chunk was popped).
+    // Outside the union: the synchronous sub-round lists overwrite the union.
+    unsigned long long qword[kQCap];
     int32_t lcnt[2];
     int32_t larc[2];
     int32_t lphase;      // local arcs accepted this phase
@@ -249,7 +264,7 @@ struct Smem {
     int32_t bloom_on;
     Ctrl ctrl;
     Snap snap;
-    int32_t qhead, qtail, qpend, qepoch;
+    int32_t qhead, qtail, qpend, qpad;
     unsigned long long qwalked;
     uint32_t bloom[kBloomWords];
 };
@@ -410,6 +425,12 @@ __device__ __forceinline__ void block_excl_scan2(Smem &sm, unsigned long long q,
     re = sm.scan_q2[wib] + (ri - r);
 }
 
+// async chunk-queue words (Smem::qword)
+__device__ __forceinline__ unsigned long long qword_pack(int64_t beg, int len)
+{
+    return (1ULL << 63) | ((unsigned long long)(len - 1) << 34) | (unsigned long long)beg;
+}
+
 // ------------------------------------------------------------ warp stages
 // Global queue: one packed atomic reserves slots and their arc range.
 __device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
@@ -536,10 +557,10 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
     const int32_t dd[4] = {d0, d1, d2, d3};
     const int64_t bb[4] = {b0, b1, b2, b3};
     unsigned bal[4];
-    int off[4], tot = 0;
+    int off[4], pre[4], tot = 0;
 #pragma unroll
     for (int r = 0; r < 4; r++) {
-        bal[r] = __ballot_sync(kFull, (wm >> r) & 1u);
+        pre[r] = ballot_excl((wm >> r) & 1u, bal[r]);  // Fig. 8(c)
         off[r] = tot;
         tot += __popc(bal[r]);
     }
@@ -550,7 +571,7 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
         base = __shfl_sync(kFull, base, 0);
 #pragma unroll
         for (int r = 0; r < 4; r++)
-            if ((wm >> r) & 1u) A.order[base + off[r] + __popc(bal[r] & lt)] = vv[r];
+            if ((wm >> r) & 1u) A.order[base + off[r] + pre[r]] = vv[r];
     } else if (lane == 0) {
         atomicAdd(&sm.removed, tot);
     }
@@ -590,7 +611,7 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
         if (lane == 0) {
             const int op = atomicAdd(&sm.lphase, sumd);
             if (op + sumd <= sm.bud_phase) {
-                int t = *(volatile int *)&sm.qtail;
+                int t = atomicAdd(&sm.qtail, 0);
                 while (t + tot <= kQCap) {
                     const int o2 = atomicCAS(&sm.qtail, t, t + tot);
                     if (o2 == t) { ok = 1; base = t; break; }
@@ -603,15 +624,10 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
         base = __shfl_sync(kFull, base, 0);
         if (ok) {
             int pos = base + incl - mine;
-            const int ep = sm.qepoch;
 #pragma unroll
             for (int r = 0; r < 4; r++) {
-                for (int q = 0; q < nc[r]; q++, pos++) {
-                    sm.qbeg[pos] = bb[r] + (int64_t)q * kBatch;
-                    sm.qlen[pos] = min(kBatch, dd[r] - q * kBatch);
-                    __threadfence_block();
-                    *(volatile int32_t *)&sm.qflag[pos] = ep;
-                }
+                for (int q = 0; q < nc[r]; q++, pos++)
+                    atomicExch(&sm.qword[pos], qword_pack(bb[r] + (int64_t)q * kBatch, min(kBatch, dd[r] - q * kBatch)));
             }
             lm = cm;
         }
@@ -841,6 +857,98 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
     }
 }
 
+// Heavy HUB walk with NON-returning decrements (Ctrl::red): arcs [a0,a1) of
+// global-queue entries [s,e) (arc prefix gq_arc, row begin gq_beg; the last
+// entry ends at arc ae).  Every target that passes the alive filter takes
+// `red.global.add -1` (Alg. 3 l.21 without its return value); nothing is
+// claimed here.  The phase that follows is a rescan -- a LEVEL phase at the
+// same k -- which claims every alive vertex this walk took to <= k (the scan
+// test deg <= k, reading R10), so each removal stays exactly-once and the
+// level-skip bound stays a lower bound (the rescan's min covers every target
+// decremented here).  With no return to wait for, a warp keeps
+// 32 x KC_RED_UNROLL arcs of colidx in flight and the next batch's loads are
+// issued before this batch's decrements.
+__device__ __forceinline__ void red_dec(int32_t *p)
+{
+    asm volatile("red.global.add.s32 [%0], -1;" ::"l"(p) : "memory");
+}
+
+__device__ void walk_red(const KArgs &A, Smem &sm, int64_t s, int64_t e, int64_t ae, int64_t a0, int64_t a1,
+                         bool use_bloom)
+{
+    constexpr int U = KC_RED_UNROLL;
+    constexpr int RB = 32 * U;
+    const int lane = threadIdx.x & 31;
+    int64_t lo = s, hi = e;
+    while (true) {  // first entry: largest i in [s,e) with P(i) <= a0 (32-ary search)
+        const int64_t step = hi - lo > 32 ? (hi - lo + 31) / 32 : 1;
+        const int64_t p = lo + lane * step;
+        bool ok = false;
+        if (p < hi) ok = ld_cg_i64(A.gq_arc + p) <= a0;
+        const unsigned b = __ballot_sync(kFull, ok);
+        lo = lo + (31 - __clz(b)) * step;
+        if (step == 1) break;
+        hi = min(hi, lo + step);
+    }
+    int64_t i = lo, a = a0;
+    while (a < a1) {
+        const int64_t j = i + lane;
+        int64_t wq = LLONG_MAX, wbeg = 0;
+        if (j < e) { wq = ld_cg_i64(A.gq_arc + j); wbeg = ld_cg_i64(A.gq_beg + j); }
+        int64_t nxt = __shfl_down_sync(kFull, wq, 1);
+        if (j + 1 >= e) nxt = ae;
+        else if (lane == 31) nxt = ld_cg_i64(A.gq_arc + j + 1);
+        const int64_t limit = min(a1, __shfl_sync(kFull, nxt, 31));
+        const int64_t bmq = wbeg - wq;
+        auto gather = [&](int64_t ab, int32_t *out) {
+            const int64_t rq = wq - ab;
+            const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
+            const int32_t lim = (int32_t)min((int64_t)RB, limit - ab);
+            // fast path: the whole batch lies in one entry (long rows: the usual case)
+            const unsigned le = __ballot_sync(kFull, q32 <= 0);
+            const int first = le ? 31 - __clz(le) : 0;
+            const int32_t qn = __shfl_sync(kFull, q32, min(first + 1, 31));
+            if (first == 31 || qn >= RB) {
+                const int64_t off = __shfl_sync(kFull, bmq, first) + ab;
+#pragma unroll
+                for (int r = 0; r < U; r++) {
+                    const int32_t my = r * 32 + lane;
+                    out[r] = (my < lim) ? ld_stream_i32(A.colidx + off + my) : -1;
+                }
+            } else {
+#pragma unroll
+                for (int r = 0; r < U; r++) {
+                    const int32_t my = r * 32 + lane;
+                    int pos = 0;
+#pragma unroll
+                    for (int bs = 16; bs >= 1; bs >>= 1) {
+                        const int32_t q = __shfl_sync(kFull, q32, pos + bs);
+                        if (q <= my) pos += bs;
+                    }
+                    const int64_t off = __shfl_sync(kFull, bmq, pos);
+                    out[r] = (my < lim) ? ld_stream_i32(A.colidx + off + ab + my) : -1;
+                }
+            }
+        };
+        int32_t un[U];
+        if (a < limit) gather(a, un);
+        while (a < limit) {
+            int32_t u[U];
+#pragma unroll
+            for (int r = 0; r < U; r++) u[r] = un[r];
+            const int64_t an = a + RB;
+            if (an < limit) gather(an, un);
+#pragma unroll
+            for (int r = 0; r < U; r++) {
+                if (u[r] >= 0 && (!use_bloom || bloom_maybe(sm, (uint32_t)u[r]))) red_dec(A.deg + u[r]);
+            }
+            a = an;
+        }
+        a = limit;
+        i += 32;
+    }
+}
+
 // Drain this CTA's local frontier (list `cur`) breadth-first with CTA-local
 // sub-rounds.  Returns the number of arcs walked.
 __device__ int64_t local_drain(const KArgs &A, Smem &sm, const int k, int cur, bool use_bloom, bool atom_only,
@@ -910,25 +1018,21 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
 {
     const int lane = threadIdx.x & 31;
     const uint64_t pol = deg_policy();
-    const int ep = sm.qepoch;
     int64_t walked = 0;
     while (true) {
-        int idx = 0;
+        unsigned long long w = 0ULL;
         if (lane == 0) {
-            idx = atomicAdd(&sm.qhead, 1);
-            if (idx >= kQCap) {
-                idx = -1;
-            } else {
-                while (*(volatile int32_t *)&sm.qflag[idx] != ep) {
-                    if (*(volatile int32_t *)&sm.qpend == 0) { idx = -1; break; }
+            const int idx = atomicAdd(&sm.qhead, 1);
+            if (idx < kQCap) {
+                while ((w = atomicExch(&sm.qword[idx], 0ULL)) == 0ULL) {
+                    if (atomicAdd(&sm.qpend, 0) == 0) break;
                 }
             }
         }
-        idx = __shfl_sync(kFull, idx, 0);
-        if (idx < 0) break;
-        __threadfence_block();
-        const int64_t beg = sm.qbeg[idx];
-        const int len = sm.qlen[idx];
+        w = __shfl_sync(kFull, w, 0);
+        if (w == 0ULL) break;
+        const int64_t beg = (int64_t)(w & ((1ULL << 34) - 1ULL));
+        const int len = (int)((w >> 34) & 127ULL) + 1;
         int32_t u[kUnroll];
 #pragma unroll
         for (int r = 0; r < kUnroll; r++) {
@@ -981,13 +1085,7 @@ __device__ int64_t drain(const KArgs &A, Smem &sm, const int k, bool use_bloom, 
         const int64_t chunks = (int64_t)sm.tot_q, arcs = (int64_t)sm.tot_q2;
         if (L > 0 && arcs >= (int64_t)KC_ASYNC_MINAVG * L && chunks <= kQCap) {
             __syncthreads();  // everyone holds its list entry: the queue may overwrite the lists
-            const int ep = sm.qepoch;
-            for (int q = 0; q < nc; q++) {
-                const int pos = (int)tq + q;
-                sm.qbeg[pos] = b + (int64_t)q * kBatch;
-                sm.qlen[pos] = min(kBatch, d - q * kBatch);
-                sm.qflag[pos] = ep;
-            }
+            for (int q = 0; q < nc; q++) sm.qword[(int)tq + q] = qword_pack(b + (int64_t)q * kBatch, min(kBatch, d - q * kBatch));
             (void)v;
             if (threadIdx.x == 0) { sm.qtail = (int)chunks; sm.qpend = (int)chunks; sm.qhead = 0; }
             __syncthreads();
@@ -1053,8 +1151,8 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
     const int lane = threadIdx.x & 31;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    if (threadIdx.x == 0) { sm.removed = 0; sm.qepoch = 0; }
-    for (int i = threadIdx.x; i < kQCap; i += kBlock) sm.qflag[i] = -1;
+    if (threadIdx.x == 0) sm.removed = 0;
+    for (int i = threadIdx.x; i < kQCap; i += kBlock) sm.qword[i] = 0ULL;
     __syncthreads();
     // The 0-shell is the isolated vertices: nothing can reach them, so
     // they are removed here -- claim bit set, core 0, counted as removed -- and
@@ -1235,7 +1333,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.bud_hub = kHub;
         sm.bud_sub = kSub;
         sm.bud_phase = kPhase;
-        sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qepoch++; sm.qwalked = 0ULL;
+        sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qwalked = 0ULL;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
@@ -1278,11 +1376,21 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
         sm.bud_hub = kHub;
         sm.bud_sub = kSub;
         sm.bud_phase = kPhase;
-        sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qepoch++; sm.qwalked = 0ULL;
+        sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qwalked = 0ULL;
     }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
     const bool bl = want_bloom(A, c, sm, cta_arcs);
+    if (c.red) {  // non-returning walk; the next phase rescans (advance())
+        const int64_t ra0 = c.as + gw * C;
+        if (ra0 < c.ae) walk_red(A, sm, c.s, c.e, c.ae, ra0, min(ra0 + C, c.ae), bl);
+        __syncthreads();
+        cta_time(A, c, 1);
+        cta_time(A, c, 2);
+        cta_count(A, c, 5, cta_arcs);
+        if (threadIdx.x == 0 && cta_arcs > 0) atomicAdd(&A.S->arcs_walked, (unsigned long long)cta_arcs);
+        return;
+    }
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_HUB;
     const int64_t a0 = c.as + gw * C;
     if (a0 < c.ae)
@@ -1343,6 +1451,23 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
             if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
             c.phase = PH_DONE;
             c.solo = 0;
+            c.red = 0;
+            return;
+        }
+        if (c.phase == PH_HUB && c.red) {
+            // after a non-returning walk: rescan the alive list at the SAME k
+            // (same level; its claims and min complete what the walk started)
+            c.red = 0;
+            const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
+            const int64_t live = p.n - removed;
+            c.phase = PH_LEVEL;
+            c.src_sel = c.alive_sel;
+            c.src_single = c.alive_single;
+            c.src_len = src_len;
+            c.compact = (live * KC_COMPACT_D < src_len * (KC_COMPACT_D - 1)) ? 1 : 0;
+            c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
+            c.solo = src_len <= (int64_t)p.solo_scan;
+            if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
             return;
         }
         if (gcnt > c.gq_cnt) {  // hub / overflow vertices pending: HUB phase
@@ -1350,6 +1475,9 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
             c.s = c.gq_cnt; c.e = gcnt; c.as = c.gq_arc; c.ae = garc;
             c.gq_cnt = gcnt; c.gq_arc = garc;
             c.solo = (c.ae - c.as) <= (int64_t)p.solo_arcs;
+            const int64_t live = p.n - removed;
+            c.red = (KC_RED_MIN > 0 && !c.solo && p.red && c.ae - c.as >= (int64_t)KC_RED_MIN &&
+                     live * KC_RED_RATIO <= c.ae - c.as) ? 1 : 0;
             return;
         }
         // level end
@@ -1596,9 +1724,8 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(const __grid_constant__ KAr
         sm.bloom_on = 0;
         sm.bloom_level = -1;
         sm.seg_cache_ok[0] = sm.seg_cache_ok[1] = 0;
-        sm.qepoch = 0;
     }
-    for (int i = threadIdx.x; i < kQCap; i += kBlock) sm.qflag[i] = -1;
+    for (int i = threadIdx.x; i < kQCap; i += kBlock) sm.qword[i] = 0ULL;
     __syncthreads();
     const Ctrl &c = sm.ctrl;
     if (c.phase == PH_INIT) phase_init(A, sm);
@@ -1626,7 +1753,7 @@ __global__ void k_l2_release(const char *base, int64_t lines)
         asm volatile("applypriority.global.L2::evict_normal [%0], 128;" ::"l"(base + i * 128) : "memory");
 }
 
-__global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan, int32_t bloom,
+__global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan, int32_t bloom, int32_t red,
                              int64_t *trace, int64_t *trace_cta, int64_t trace_cap)
 {
     if (threadIdx.x == 0 && blockIdx.x == 0) {
@@ -1645,6 +1772,7 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
         S->prm.solo_arcs = solo_arcs;
         S->prm.solo_scan = solo_scan;
         S->prm.bloom = bloom;
+        S->prm.red = red;
         S->trace = trace;
         S->trace_cta = trace_cta;
         S->trace_cap = trace ? trace_cap : 0;

@@ -201,6 +201,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     int64_t *trace = opt ? opt->trace_out : nullptr;
     const int64_t trace_cap = (opt && opt->trace_out) ? opt->trace_cap : 0;
     const int bloom = (opt && (opt->flags & KCORE_FLAG_NO_BLOOM)) ? 0 : 1;
+    const int red = (opt && (opt->flags & KCORE_FLAG_NO_RED)) ? 0 : 1;
     const size_t smem = sizeof(Smem);
 
     const size_t need = carve(nullptr, n, nullptr);
@@ -244,7 +245,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaEventCreate(&ev0));
         KC_CUDA(cudaEventCreate(&ev1));
     }
-    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, trace,
+    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, red, trace,
                                    trace ? opt->trace_cta_out : nullptr, trace_cap);
     KC_CUDA(cudaGetLastError());
     if (stats) KC_CUDA(cudaEventRecord(ev0, st));

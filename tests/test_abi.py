@@ -26,6 +26,12 @@ def test_library_exports_every_declared_symbol():
     assert set(names) == set(kc.EXPORTS)
 
 
+def test_library_exports_test_hooks():
+    lib = kc.library()
+    for name in _declared("kcore_test.h"):
+        assert hasattr(lib, name), name
+
+
 def test_generator_library_exports():
     import kcgen
     lib = kcgen._load()
