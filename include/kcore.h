@@ -76,6 +76,9 @@ typedef enum {
                                 /* (default: phases walking >= 2^21 arcs over an alive set */
                                 /* <= 1/8 of them use non-returning red.global.add and a   */
                                 /* rescan of the alive list at the same k)      */
+#define KCORE_FLAG_NO_NEAR 8    /* ablation: every level scans the whole alive list       */
+                                /* (default: long alive lists hand the next levels a near */
+                                /* list of the vertices with degree <= k + W)  */
 
 /* Algorithms selectable through kcore_options.algo. */
 #define KCORE_ALGO_PERSISTENT 0 /* default: one persistent kernel, device-resident loop */
@@ -106,7 +109,9 @@ typedef struct {
                              /* walk, end of local drain, barrier arrival, local sub-  */
                              /* rounds, arcs walked, vertices removed, largest sub-     */
                              /* round in arcs}                                          */
-    int64_t reserved[1];
+    int32_t near_min_alive;  /* > 0: alive-list length from which level scans build a   */
+                             /* near list (default 2^17; tuning / tests)                 */
+    int32_t near_window;     /* > 0: initial near window W (default 16; tuning / tests)  */
 } kcore_options;
 
 /* Run statistics (filled when a non-NULL pointer is passed; this makes the
@@ -126,7 +131,9 @@ typedef struct {
     int32_t trace_len;     /* trace records written (see kcore_options.trace_out)    */
     double kernel_ms;      /* device time of the decomposition kernel(s) (CUDA events) */
     int64_t launches;      /* kernels this call launched                              */
-    int64_t reserved[2];
+    int64_t near_scans;    /* level scans that read the near list instead of the     */
+                           /* whole alive list (included in `scanned`)               */
+    int64_t reserved[1];
 } kcore_stats;
 
 /* Core decomposition on one GPU (north-star signature).  All array pointers

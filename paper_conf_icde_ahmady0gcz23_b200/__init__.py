@@ -40,6 +40,7 @@ ALGO_HOSTLOOP = 1
 FLAG_NO_BLOOM = 1
 FLAG_NO_L2_PERSIST = 2
 FLAG_NO_RED = 4
+FLAG_NO_NEAR = 8
 
 # every symbol include/kcore.h declares (checked by tests/test_abi.py)
 EXPORTS = (
@@ -63,7 +64,7 @@ class _Options(ctypes.Structure):
         ("order_out", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
         ("workspace_bytes", ctypes.c_size_t), ("trace_out", ctypes.c_void_p),
         ("trace_cap", ctypes.c_int64), ("flags", ctypes.c_int32), ("reserved1", ctypes.c_int32),
-        ("trace_cta_out", ctypes.c_void_p), ("reserved", ctypes.c_int64 * 1),
+        ("trace_cta_out", ctypes.c_void_p), ("near_min_alive", ctypes.c_int32), ("near_window", ctypes.c_int32),
     ]
 
 
@@ -75,7 +76,7 @@ class _Stats(ctypes.Structure):
         ("compactions", ctypes.c_int64), ("hub_arcs", ctypes.c_int64), ("kmax", ctypes.c_int32),
         ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
         ("trace_len", ctypes.c_int32), ("kernel_ms", ctypes.c_double),
-        ("launches", ctypes.c_int64), ("reserved", ctypes.c_int64 * 2),
+        ("launches", ctypes.c_int64), ("near_scans", ctypes.c_int64), ("reserved", ctypes.c_int64 * 1),
     ]
 
 
@@ -95,12 +96,13 @@ class Stats:
     kernel_ms: float
     trace_len: int = 0
     launches: int = 0
+    near_scans: int = 0
 
     @classmethod
     def _from(cls, s: _Stats) -> "Stats":
         return cls(s.levels, s.phases, s.solo_phases, s.barriers, s.scanned, s.arcs_walked,
                    s.compactions, s.hub_arcs, s.kmax, s.grid_blocks, s.block_threads, s.kernel_ms,
-                   s.trace_len, s.launches)
+                   s.trace_len, s.launches, s.near_scans)
 
 
 _lib = None
@@ -180,7 +182,8 @@ def _check_csr_tensors(rowptr, colidx):
 def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=None,
                     algo: int = ALGO_PERSISTENT, blocks_per_sm: int = 0, solo_arcs: int = 0,
                     solo_scan: int = 0, bloom: bool = True, trace=None,
-                    trace_cta=None, stats: bool = False, l2_persist: bool = True, red: bool = True):
+                    trace_cta=None, stats: bool = False, l2_persist: bool = True, red: bool = True,
+                    near: bool = True, near_min_alive: int = 0, near_window: int = 0):
     """Core numbers of the graph (rowptr int64[n+1], colidx int32[m] CUDA tensors).
 
     Runs on the current stream of the tensors' device.  Returns an int32 tensor
@@ -199,8 +202,8 @@ def kcore_decompose(rowptr, colidx, *, core_out=None, order_out=None, workspace=
                    trace.data_ptr() if trace is not None else None,
                    trace.shape[0] if trace is not None else 0,
                    (0 if bloom else FLAG_NO_BLOOM) | (0 if l2_persist else FLAG_NO_L2_PERSIST) |
-                   (0 if red else FLAG_NO_RED), 0,
-                   trace_cta.data_ptr() if trace_cta is not None else None)
+                   (0 if red else FLAG_NO_RED) | (0 if near else FLAG_NO_NEAR), 0,
+                   trace_cta.data_ptr() if trace_cta is not None else None, near_min_alive, near_window)
     st = _Stats()
     with torch.cuda.device(dev):
         rc = _load().kcore_decompose_ex(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,

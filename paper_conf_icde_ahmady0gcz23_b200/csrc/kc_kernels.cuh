@@ -128,9 +128,6 @@ constexpr int kTraceFields = 8;
 #ifndef KC_FASTSUB
 #define KC_FASTSUB 1
 #endif
-#ifndef KC_TAGBAR
-#define KC_TAGBAR 0  // 1: grid barrier publishes the snapshot as generation-tagged words (no release flag)
-#endif
 #ifndef KC_AO_HUB
 #define KC_AO_HUB 1
 #endif
@@ -153,6 +150,22 @@ constexpr int kTraceFields = 8;
 #ifndef KC_RED_UNROLL
 #define KC_RED_UNROLL 8
 #endif
+// Near list: a FULL level scan over an alive list of at
+// least KC_NEAR_MIN_A entries also collects every alive vertex with
+// k < deg <= theta = k + W into a near list, and walks append a vertex when its
+// decrement crosses theta+1 -> theta.  Levels k' <= theta then scan only the
+// near list: every alive vertex of degree <= theta is in it, so the frontier
+// (deg <= k') and the level-skip bound min(near min, walk min, theta+1) are
+// exact.  W adapts per epoch (KC_NEAR_W initial).  0 disables.
+#ifndef KC_NEAR_MIN_A
+#define KC_NEAR_MIN_A (1 << 17)
+#endif
+#ifndef KC_NEAR_W
+#define KC_NEAR_W 16
+#endif
+#ifndef KC_NEAR
+#define KC_NEAR 1  // 0: compile the near list out (walks never test for theta crossings)
+#endif
 enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
 struct Ctrl {
@@ -160,9 +173,9 @@ struct Ctrl {
     int32_t compact, src_sel, dst_sel, alive_sel;
     int32_t src_single, alive_single;  // 1: the list is one contiguous run in segment 0
     int32_t red;                       // HUB phase walks with non-returning decrements (then a rescan)
-    int32_t pad1;
+    int32_t near_app;                  // walks append theta+1 -> theta crossings to near[near_app] (-1: off)
     int64_t arcs_lvl0;                 // arcs walked when the level began
-    int64_t pad2;
+    int64_t st_near;                   // near-list level scans
     int64_t src_len, alive_len;
     int64_t s, e, as, ae;          // HUB: global-queue slots [s,e), arcs [as,ae)
     int64_t gq_cnt, gq_arc;        // global queue consumed so far
@@ -170,6 +183,17 @@ struct Ctrl {
     int64_t level;                 // level index (for the Bloom cache)
     int64_t st_levels, st_phases, st_solo, st_bar, st_scanned, st_compact, st_hubarcs;
     int32_t st_kmax, st_pad;
+    // near-list state (KC_NEAR_MIN_A)
+    int32_t near_on;     // an epoch is active: every alive vertex with deg <= theta is in near[near_cur]
+    int32_t theta;
+    int32_t near_cur;    // buffer holding the list the next near scan reads
+    int32_t near_scan;   // this LEVEL phase scans near[near_cur] (compacting into near[near_cur ^ 1])
+    int32_t near_build;  // this FULL LEVEL phase also collects k < deg <= theta into near[near_cur ^ 1]
+    int32_t near_reset;  // buffer whose tail the barrier after this phase resets (-1: none)
+    int32_t near_w;      // window W of the next epoch
+    int32_t near_lv;     // near levels in the current epoch
+    int64_t near_len;    // entries of near[near_cur] when this phase began
+    int64_t near_first;  // near-list length at the epoch's first near scan
 };
 
 static_assert(sizeof(Ctrl) % 16 == 0, "Ctrl is copied as int4");
@@ -179,6 +203,7 @@ struct Snap {
     unsigned long long gq;         // packed global-queue tail
     unsigned long long ord;        // order tail (= removed vertices)
     unsigned long long alive_out;  // compaction output length
+    unsigned long long near[2];    // near-list tails
     int32_t min;
     int32_t pad;
 };
@@ -188,7 +213,10 @@ struct Params {
     int32_t solo_arcs;  // HUB phases with <= this many arcs run solo
     int32_t solo_scan;  // LEVEL phases over <= this many entries run solo
     int32_t bloom;      // 0 disables the Bloom filter
-    int32_t red;        // 0 disables non-returning heavy HUB walks (KC_RED_MIN)
+    int16_t red;        // 0 disables non-returning heavy HUB walks (KC_RED_MIN)
+    int16_t near;       // 0 disables the near list (KC_NEAR_MIN_A)
+    int32_t near_min;   // alive-list length from which a FULL scan builds a near list
+    int32_t near_w;     // initial near window W
 };
 
 struct State {
@@ -199,8 +227,8 @@ struct State {
     alignas(128) uint32_t bar_count;            // grid barrier arrivals (monotone)
     alignas(128) uint32_t bar_gen;              // grid barrier generation
     Snap snap[2];                               // counters at barrier gen, by gen & 1
-    alignas(128) unsigned long long tsnap[8];   // KC_TAGBAR: (gen & 0xffff) << 48 | value, see grid_barrier
     alignas(128) unsigned long long arcs_walked;
+    alignas(128) unsigned long long near_tail[2];  // near-list append cursors (one line)
     alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
     alignas(128) Params prm;
     int64_t *trace;                             // optional [trace_cap][kTraceFields]
@@ -220,6 +248,7 @@ struct KArgs {
     int64_t *gq_beg;
     int64_t *gq_arc;
     int32_t *alive[2];  // alive lists, partitioned into nseg per-CTA segments
+    int32_t *near[2];   // near lists (contiguous runs, global cursors S->near_tail)
     int32_t *seg_len[2];  // entries of segment b in alive[x]: seg_len[x][b]
     int64_t seg_R;        // segment region size: segment b lives at [b*R, b*R + len)
     int32_t nseg;         // = persistent grid size
@@ -264,7 +293,8 @@ struct Smem {
     int32_t bloom_on;
     Ctrl ctrl;
     Snap snap;
-    int32_t qhead, qtail, qpend, qpad;
+    int32_t qhead, qtail, qpend;
+    int32_t near_th1;  // theta + 1 while walks feed a near list, else INT_MIN (set per phase)
     unsigned long long qwalked;
     uint32_t bloom[kBloomWords];
 };
@@ -433,7 +463,15 @@ __device__ __forceinline__ unsigned long long qword_pack(int64_t beg, int len)
 
 // ------------------------------------------------------------ warp stages
 // Global queue: one packed atomic reserves slots and their arc range.
-__device__ __noinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
+#ifndef KC_GQF_INLINE
+#define KC_GQF_INLINE 0  // the global-queue flush is a rare path: out of line keeps the kernel small
+#endif
+#if KC_GQF_INLINE
+__device__ __forceinline__
+#else
+__device__ __noinline__
+#endif
+void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
     if (gcnt == 0) return;
@@ -693,6 +731,27 @@ __device__ __forceinline__ bool claim(const KArgs &A, int32_t v)
     return (atom_or_claim(A.claimed + (v >> 5), bit, deg_policy()) & bit) == 0u;
 }
 
+// theta+1 of the running near epoch (INT_MIN: no near list), re-read from
+// shared memory at each use so it never holds a register across the walk loop
+__device__ __forceinline__ int near_th1(const Smem &sm)
+{
+    if (!KC_NEAR) return INT_MIN;
+    return *(const volatile int32_t *)&sm.near_th1;
+}
+
+// One theta+1 -> theta crossing joins the near list: a lane-level append (each
+// vertex crosses once per epoch, so these are rare; no warp-collective code in
+// the walk's hot loop).
+__device__ __forceinline__ void near_push(const KArgs &A, const Smem &sm, int32_t u)
+{
+    const int app = *(const volatile int32_t *)&sm.ctrl.near_app;
+    const unsigned long long pos = atomicAdd(&A.S->near_tail[app], 1ULL);
+    A.near[app][pos] = u;
+}
+
+// Near list: targets whose decrement crossed theta+1 -> theta (cm bit r set for
+// u[r]) join near[near_app] -- one warp-aggregated append.  Each vertex crosses
+// once per epoch (degrees only decrease), so the list stays within n.
 // --------------------------------------------------------- arc walking
 // Hits of one batch (u reached k): claim, fetch row bounds, prefetch the
 // row's first line for the next hop, route.  Out of line: rare path.
@@ -841,14 +900,17 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
             unsigned hm = 0;
+            const int th1 = near_th1(sm);
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
                 if (old[r] == k + 1) hm |= 1u << r;
-                else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
+                else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
             }
             const unsigned hb = __ballot_sync(kFull, hm != 0);
             if (lane == 0) PROBE_W(11, (threadIdx.x >> 5) | ((int64_t)__popc(hb) << 8) | ((int64_t)old[0] << 16));
-            if (hb) handle_hits(A, sm, k, nx, u[0], u[1], u[2], u[3], hm, gcnt);
+            if (hb) {
+                handle_hits(A, sm, k, nx, u[0], u[1], u[2], u[3], hm, gcnt);
+            }
             if (lane == 0) PROBE_W(12, threadIdx.x >> 5);
             a = an;
         }
@@ -1051,12 +1113,15 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
             old[r] = d > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
         }
         unsigned hm = 0;
+        const int th1 = near_th1(sm);
 #pragma unroll
         for (int r = 0; r < kUnroll; r++) {
             if (old[r] == k + 1) hm |= 1u << r;
-            else if (old[r] > k + 1) lmin = min(lmin, old[r] - 1);
+            else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
         }
-        if (__any_sync(kFull, hm != 0)) handle_hits(A, sm, k, kAsyncNx, u[0], u[1], u[2], u[3], hm, gcnt);
+        if (__any_sync(kFull, hm != 0)) {
+            handle_hits(A, sm, k, kAsyncNx, u[0], u[1], u[2], u[3], hm, gcnt);
+        }
         walked += len;
         __syncwarp();
         if (lane == 0) atomicSub(&sm.qpend, 1);
@@ -1195,7 +1260,8 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
 // min for the level skip and, when compacting, ballot compaction (Fig. 8(c))
 // into dst[0..) with a shared-memory cursor.  No block sync, no global atomics.
 __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_t *src, int64_t lo,
-                           int64_t hi, int32_t *dst, int &lmin, int &gcnt)
+                           int64_t hi, int32_t *dst, int &lmin, int &gcnt, int32_t *ndst = nullptr,
+                           unsigned long long *ntail = nullptr)
 {
     const int k = c.k;
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -1233,6 +1299,28 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
             if (vv[j] < 0) continue;
             if (dd[j] <= k) { if (k == 0 || claim(A, vv[j])) wm |= 1u << j; }
             else if (dd[j] > k) { lmin = min(lmin, dd[j]); km |= 1u << j; }
+        }
+        if (ndst) {  // near list: k < deg <= theta (a near scan's compaction, or a build)
+            unsigned nm = 0;
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++)
+                if (((km >> j) & 1u) && dd[j] <= c.theta) nm |= 1u << j;
+            const int mine = __popc(nm);
+            int incl = mine;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(kFull, incl, o);
+                if (lane >= o) incl += t;
+            }
+            const int tot = __shfl_sync(kFull, incl, 31);
+            if (tot) {
+                unsigned long long pos = 0;
+                if (lane == 31) pos = atomicAdd(ntail, (unsigned long long)tot);
+                pos = __shfl_sync(kFull, pos, 31) + (unsigned long long)(incl - mine);
+#pragma unroll
+                for (int j = 0; j < kScanItems; j++)
+                    if ((nm >> j) & 1u) ndst[pos++] = vv[j];
+            }
         }
         if (dst) {
             int mine = __popc(km), incl = mine;
@@ -1286,6 +1374,19 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
                            int &gcnt)
 {
     const bool solo = (nblk == 1);
+    int32_t *ndst = nullptr;
+    unsigned long long *ntail = nullptr;
+    if (c.near_scan || c.near_build) {
+        ndst = A.near[c.near_cur ^ 1];
+        ntail = &A.S->near_tail[c.near_cur ^ 1];
+    }
+    if (c.near_scan) {  // the near list: one contiguous run, an even slice per CTA, no alive compaction
+        const int64_t L = c.near_len;
+        const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
+        scan_range(A, c, sm, A.near[c.near_cur], lo, hi, nullptr, lmin, gcnt, ndst, ntail);
+        __syncthreads();
+        return;
+    }
     const int32_t *srcb = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
     int32_t *dstb = c.compact ? A.alive[c.dst_sel] : nullptr;
     const int dseg = solo ? 0 : bid;
@@ -1296,15 +1397,15 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
         // contiguous source of c.src_len entries: an even slice per CTA
         const int64_t L = c.src_len;
         const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
-        scan_range(A, c, sm, srcb, lo, hi, dst, lmin, gcnt);
+        scan_range(A, c, sm, srcb, lo, hi, dst, lmin, gcnt, ndst, ntail);
     } else if (!solo) {
         // this CTA wrote its own segment's length at the last compaction
         const int64_t len = sm.seg_cache_ok[c.src_sel] ? sm.seg_cache[c.src_sel] : ld_cg_i32(A.seg_len[c.src_sel] + bid);
-        scan_range(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt);
+        scan_range(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
     } else {
         for (int b = 0; b < A.nseg; b++) {
             const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
-            if (len) scan_range(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, gcnt);
+            if (len) scan_range(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
         }
     }
     __syncthreads();
@@ -1334,6 +1435,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.bud_sub = kSub;
         sm.bud_phase = kPhase;
         sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qwalked = 0ULL;
+        sm.near_th1 = c.near_app >= 0 ? c.theta + 1 : INT_MIN;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
@@ -1377,6 +1479,7 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
         sm.bud_sub = kSub;
         sm.bud_phase = kPhase;
         sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qwalked = 0ULL;
+        sm.near_th1 = c.near_app >= 0 ? c.theta + 1 : INT_MIN;
     }
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
@@ -1394,8 +1497,8 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_HUB;
     const int64_t a0 = c.as + gw * C;
     if (a0 < c.ae)
-        walk<false>(A, sm, c.k, 0, KC_ASYNC == 1 ? kAsyncNx : 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin, gcnt,
-                    KC_CF_HUB);
+        walk<false>(A, sm, c.k, 0, KC_ASYNC == 1 ? kAsyncNx : 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin,
+                    gcnt, KC_CF_HUB);
     int64_t walked = cta_arcs;
     __syncthreads();
     cta_time(A, c, 1);
@@ -1416,13 +1519,67 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
 // ---------------------------------------------------------------- control
 // The pure transition function (Alg. 1 l.5-9 and the level skip).  Every CTA
 // applies it to identical inputs, so all copies stay identical.
+// A FULL level scan (the alive list) at c.k.  With the near list enabled and
+// a long alive list it also collects the next epoch's near list.
+__device__ __forceinline__ void setup_full(Ctrl &c, const Params &p, int64_t removed)
+{
+    const int64_t live = p.n - removed;
+    const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
+    c.phase = PH_LEVEL;
+    c.src_sel = c.alive_sel;
+    c.src_single = c.alive_single;
+    c.src_len = src_len;
+    c.compact = (live * KC_COMPACT_D < src_len * (KC_COMPACT_D - 1)) ? 1 : 0;  // >= 1/D of the source is dead
+    c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
+    c.solo = src_len <= (int64_t)p.solo_scan;
+    // a solo scan of a segmented list gathers it into one run for next time
+    if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
+    c.near_scan = 0;
+    if (KC_NEAR && p.near && !c.solo && src_len >= (int64_t)p.near_min && c.near_w > 0) {
+        c.near_build = 1;
+        c.near_on = 1;
+        c.theta = (int32_t)min((int64_t)INT_MAX - 2, (int64_t)c.k + c.near_w);
+        c.near_app = c.near_cur ^ 1;  // scan and walks of this phase fill the other buffer
+        c.near_reset = c.near_cur;    // the previous epoch's list is dropped at this barrier
+        c.near_lv = 0;
+        c.near_first = 0;
+    } else {
+        c.near_build = 0;
+        c.near_on = 0;
+        c.near_app = -1;
+        c.near_reset = -1;
+    }
+}
+
+// A near level scan at c.k <= theta: reads near[near_cur], compacts into the other buffer.
+__device__ __forceinline__ void setup_near(Ctrl &c, const Snap &sn, const Params &p)
+{
+    c.phase = PH_LEVEL;
+    c.near_scan = 1;
+    c.near_build = 0;
+    c.near_len = (int64_t)sn.near[c.near_cur];
+    // the alive list stays as it is (not scanned, not compacted); the Bloom
+    // filter logic keeps reading its length from src_len
+    c.src_sel = c.alive_sel;
+    c.src_single = c.alive_single;
+    c.src_len = c.alive_sel < 0 ? p.n : c.alive_len;
+    c.compact = 0;
+    c.solo = 0;
+    c.near_app = c.near_cur ^ 1;
+    c.near_reset = c.near_cur;
+    if (c.near_lv == 0) c.near_first = c.near_len;
+    c.near_lv++;
+    c.st_near++;
+}
+
+// The pure transition function (Alg. 1 l.5-9 and the level skip).  Every CTA
+// applies it to identical inputs, so all copies stay identical.
 __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
 {
     const int64_t gcnt = (int64_t)(sn.gq >> kArcBits), garc = (int64_t)(sn.gq & kArcMask);
     const int64_t removed = (int64_t)sn.ord;
     c.level_min = min(c.level_min, sn.min);
     int next_k = 0;
-    bool new_level = false;
     if (c.phase == PH_INIT) {
         if (removed > 0) { c.st_levels = 1; c.st_kmax = 0; }  // the 0-shell, removed by INIT
         if (removed >= p.n) {  // nothing but isolated vertices
@@ -1432,21 +1589,24 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         next_k = c.level_min;  // smallest positive degree
         c.level_min = INT_MAX;
         c.level = -1;
-        new_level = true;
     } else {
         c.st_phases++;
         if (c.solo) c.st_solo++;
         if (c.phase == PH_LEVEL) {
-            c.st_scanned += c.src_len;
+            c.st_scanned += c.near_scan ? c.near_len : c.src_len;
             if (c.compact) {
                 c.alive_sel = c.dst_sel;
                 c.alive_len = (int64_t)sn.alive_out;
                 c.alive_single = c.solo;  // a solo scan compacts into one run
                 c.st_compact++;
             }
+            if (c.near_scan || c.near_build) c.near_cur ^= 1;  // the list this phase wrote is current
+            c.near_scan = 0;
+            c.near_build = 0;
         } else {
             c.st_hubarcs += c.ae - c.as;
         }
+        c.near_reset = -1;
         if (removed >= p.n) {  // every vertex claimed: the rest of the level changes nothing
             if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
             c.phase = PH_DONE;
@@ -1456,18 +1616,10 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
         }
         if (c.phase == PH_HUB && c.red) {
             // after a non-returning walk: rescan the alive list at the SAME k
-            // (same level; its claims and min complete what the walk started)
+            // (same level; its claims and min complete what the walk started).
+            // The walk appended no theta crossings, so a near epoch restarts here.
             c.red = 0;
-            const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
-            const int64_t live = p.n - removed;
-            c.phase = PH_LEVEL;
-            c.src_sel = c.alive_sel;
-            c.src_single = c.alive_single;
-            c.src_len = src_len;
-            c.compact = (live * KC_COMPACT_D < src_len * (KC_COMPACT_D - 1)) ? 1 : 0;
-            c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
-            c.solo = src_len <= (int64_t)p.solo_scan;
-            if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
+            setup_full(c, p, removed);
             return;
         }
         if (gcnt > c.gq_cnt) {  // hub / overflow vertices pending: HUB phase
@@ -1478,51 +1630,53 @@ __device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
             const int64_t live = p.n - removed;
             c.red = (KC_RED_MIN > 0 && !c.solo && p.red && c.ae - c.as >= (int64_t)KC_RED_MIN &&
                      live * KC_RED_RATIO <= c.ae - c.as) ? 1 : 0;
+            c.near_app = c.near_on ? c.near_cur : -1;
             return;
         }
         // level end
         if (removed > c.ord_lvl0) { c.st_levels++; c.st_kmax = c.k; }
-        if (removed >= p.n) {
-            c.phase = PH_DONE;
-            c.solo = 0;
-            return;
-        }
         next_k = max(c.k + 1, c.level_min);
+        if (c.near_on) {
+            // vertices outside the near list have degree > theta
+            next_k = max(c.k + 1, min(c.level_min, c.theta + 1));
+        }
         c.level_min = INT_MAX;
-        new_level = true;
     }
-    if (new_level) {
-        const int64_t live = p.n - removed;
-        const int64_t src_len = c.alive_sel < 0 ? p.n : c.alive_len;
-        const bool compact = live * KC_COMPACT_D < src_len * (KC_COMPACT_D - 1);  // >= 1/D of the source is dead
-        c.phase = PH_LEVEL;
-        c.k = next_k;
-        c.level++;
-        c.src_sel = c.alive_sel;
-        c.src_single = c.alive_single;
-        c.src_len = src_len;
-        c.compact = compact ? 1 : 0;
-        c.dst_sel = c.alive_sel < 0 ? 0 : 1 - c.alive_sel;
-        c.solo = src_len <= (int64_t)p.solo_scan;
-        // a solo scan of a segmented list gathers it into one run for next time
-        if (c.solo && c.alive_sel >= 0 && !c.alive_single) c.compact = 1;
-        c.ord_lvl0 = removed;
-        c.arcs_lvl0 = (int64_t)sn.arcs;
+    // new level at next_k
+    c.k = next_k;
+    c.level++;
+    c.ord_lvl0 = removed;
+    c.arcs_lvl0 = (int64_t)sn.arcs;
+    if (c.near_on && next_k <= c.theta) {
+        setup_near(c, sn, p);
+        return;
     }
+    if (c.near_on) {  // epoch over: adapt the window to the list it produced
+        const int64_t A = c.alive_sel < 0 ? p.n : c.alive_len;
+        if (c.near_lv > 0 && c.near_first * 4 > A) c.near_w = max(1, c.near_w / 2);
+        else if (c.near_first * 32 < A) c.near_w = min(1 << 14, c.near_w * 2);
+    }
+    setup_full(c, p, removed);
 }
 
 // Snapshot + reset of the counters (caller guarantees nobody else touches them).
-__device__ __forceinline__ Snap take_snapshot(State *S, unsigned grid)
+__device__ __forceinline__ Snap take_snapshot(State *S, unsigned grid, int near_reset)
 {
     Snap sn;
     sn.arcs = ld_relaxed_u64(&S->arcs_walked);
     sn.gq = ld_relaxed_u64(&S->gq_tail);
     sn.ord = ld_relaxed_u64(&S->ord_tail);
     sn.alive_out = ld_relaxed_u64(&S->alive_out);
+    sn.near[0] = ld_relaxed_u64(&S->near_tail[0]);
+    sn.near[1] = ld_relaxed_u64(&S->near_tail[1]);
     sn.min = ld_relaxed_i32(&S->min_next);
     sn.pad = 0;
     S->alive_out = 0ULL;
     S->min_next = INT_MAX;
+    // the list this phase consumed (a near scan's source / the previous list of
+    // a build) is empty from now on; nobody appends to it until it is a scan's
+    // destination again
+    if (near_reset >= 0) S->near_tail[near_reset] = 0ULL;
     return sn;
 }
 
@@ -1545,16 +1699,6 @@ __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &s
 
 // Grid barrier; the last arriver snapshots+resets the counters.
 //
-// KC_TAGBAR: the last arriver publishes the snapshot as six 64-bit words, each
-// tagged with the new generation in its top 16 bits, after a release fence;
-// the others poll all six words at once (independent relaxed loads, one round
-// trip per poll) until every tag is the new generation, then fence (acquire).
-// No separate flag store/poll and no second read of the snapshot after the
-// flag: one memory round trip less on both sides of every barrier.  A waiter
-// of generation g finishes reading before it arrives at barrier g+1, so one
-// set of words suffices; a stale word carries tag g != g+1 (mod 2^16).
-constexpr int kTagShift = 48;
-constexpr unsigned long long kTagVal = (1ULL << kTagShift) - 1ULL;
 
 __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
 {
@@ -1571,43 +1715,8 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
         const uint32_t gen = t / (uint32_t)gridDim.x;
         PROBE(35, t);
         Snap sn;
-#if KC_TAGBAR
-        const unsigned long long tag = (unsigned long long)((gen + 1u) & 0xffffu) << kTagShift;
         if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
-            sn = take_snapshot(S, gridDim.x);
-            fence_acq_rel_gpu();  // release: everything this CTA observed before the words
-            st_relaxed_u64(&S->tsnap[0], tag | sn.ord);
-            st_relaxed_u64(&S->tsnap[1], tag | sn.alive_out);
-            st_relaxed_u64(&S->tsnap[2], tag | (unsigned long long)(uint32_t)sn.min);
-            st_relaxed_u64(&S->tsnap[3], tag | (sn.gq >> kArcBits));
-            st_relaxed_u64(&S->tsnap[4], tag | (sn.gq & kArcMask));
-            st_relaxed_u64(&S->tsnap[5], tag | sn.arcs);
-        } else {
-            unsigned long long w0, w1, w2, w3, w4, w5;
-            while (true) {
-                w0 = ld_relaxed_u64(&S->tsnap[0]);
-                w1 = ld_relaxed_u64(&S->tsnap[1]);
-                w2 = ld_relaxed_u64(&S->tsnap[2]);
-                w3 = ld_relaxed_u64(&S->tsnap[3]);
-                w4 = ld_relaxed_u64(&S->tsnap[4]);
-                w5 = ld_relaxed_u64(&S->tsnap[5]);
-                const unsigned long long hi = ~kTagVal;
-                if (((w0 & hi) == tag) & ((w1 & hi) == tag) & ((w2 & hi) == tag) & ((w3 & hi) == tag) &
-                    ((w4 & hi) == tag) & ((w5 & hi) == tag))
-                    break;
-            }
-            fence_acq_rel_gpu();  // acquire: pairs with the last arriver's fence
-            PROBE(34, 0);
-            sn.ord = w0 & kTagVal;
-            sn.alive_out = w1 & kTagVal;
-            sn.min = (int32_t)(uint32_t)(w2 & 0xffffffffULL);
-            sn.gq = ((w3 & kTagVal) << kArcBits) | (w4 & kTagVal);
-            sn.arcs = w5 & kTagVal;
-            sn.pad = 0;
-        }
-#else
-        if ((t + 1u) == (uint32_t)gridDim.x * (gen + 1u)) {
-            sn = take_snapshot(S, gridDim.x);
+            sn = take_snapshot(S, gridDim.x, sm.ctrl.near_reset);
             S->snap[(gen + 1u) & 1u] = sn;
             st_release_u32(&S->bar_gen, gen + 1u);
         } else {
@@ -1619,10 +1728,11 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
             sn.gq = ld_relaxed_u64(&ps->gq);
             sn.ord = ld_relaxed_u64(&ps->ord);
             sn.alive_out = ld_relaxed_u64(&ps->alive_out);
+            sn.near[0] = ld_relaxed_u64(&ps->near[0]);
+            sn.near[1] = ld_relaxed_u64(&ps->near[1]);
             sn.min = ld_relaxed_i32(&ps->min);
             sn.pad = 0;
         }
-#endif
         sm.snap = sn;
     }
     __syncthreads();
@@ -1643,7 +1753,7 @@ __device__ void solo_run(const KArgs &A, Smem &sm, const Params &p)
         run_phase(A, c, sm, 0, 1);  // ends with __syncthreads (block_min_atomic)
         if (threadIdx.x == 0) {
             __threadfence();
-            const Snap sn = take_snapshot(S, 1u);
+            const Snap sn = take_snapshot(S, 1u, sm.ctrl.near_reset);
             trace_rec(S, sm.ctrl, sn, 0);
             advance(sm.ctrl, sn, p);
         }
@@ -1663,6 +1773,9 @@ __device__ __forceinline__ void init_ctrl(Ctrl &z)
     z.level_min = INT_MAX;
     z.alive_sel = -1;
     z.src_sel = -1;
+    z.near_app = -1;
+    z.near_reset = -1;
+    z.near_w = 0;  // set from Params by the caller
 }
 
 __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant__ KArgs A)
@@ -1671,7 +1784,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant_
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
     State *S = A.S;
     const Params p = S->prm;
-    if (threadIdx.x == 0) init_ctrl(sm.ctrl);
+    if (threadIdx.x == 0) { init_ctrl(sm.ctrl); sm.ctrl.near_w = p.near_w; }
 #ifdef KC_PROBE
     if (threadIdx.x == 0) { s_probe_n = 0u; s_probe_k = 0; }
     __syncthreads();
@@ -1737,7 +1850,7 @@ __global__ void k_leader(const __grid_constant__ KArgs A, int32_t *phase_out)
     State *S = A.S;
     const Params p = S->prm;
     Ctrl c = S->pub;
-    const Snap sn = take_snapshot(S, gridDim.x);
+    const Snap sn = take_snapshot(S, gridDim.x, c.near_reset);
     trace_rec(S, c, sn, 1);
     c.st_bar++;
     advance(c, sn, p);
@@ -1754,6 +1867,7 @@ __global__ void k_l2_release(const char *base, int64_t lines)
 }
 
 __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t solo_scan, int32_t bloom, int32_t red,
+                             int32_t near_min, int32_t near_w,
                              int64_t *trace, int64_t *trace_cta, int64_t trace_cap)
 {
     if (threadIdx.x == 0 && blockIdx.x == 0) {
@@ -1763,16 +1877,20 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
         S->min_next = INT_MAX;
         S->bar_count = 0u;
         S->bar_gen = 0u;
-        for (int i = 0; i < 8; i++) S->tsnap[i] = 0ULL;  // tag 0: generation 0 is never awaited
         S->arcs_walked = 0ULL;
+        S->near_tail[0] = S->near_tail[1] = 0ULL;
         Ctrl z;
         init_ctrl(z);
+        z.near_w = near_w > 0 ? near_w : KC_NEAR_W;
         S->pub = z;
         S->prm.n = n;
         S->prm.solo_arcs = solo_arcs;
         S->prm.solo_scan = solo_scan;
         S->prm.bloom = bloom;
-        S->prm.red = red;
+        S->prm.red = (int16_t)(red & 1);
+        S->prm.near = (int16_t)((red >> 1) & 1);
+        S->prm.near_min = near_min > 0 ? near_min : KC_NEAR_MIN_A;
+        S->prm.near_w = near_w > 0 ? near_w : KC_NEAR_W;
         S->trace = trace;
         S->trace_cta = trace_cta;
         S->trace_cap = trace ? trace_cap : 0;

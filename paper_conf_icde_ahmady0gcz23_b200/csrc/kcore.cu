@@ -76,6 +76,7 @@ struct Carve {
     int32_t *gq_v;
     int64_t *gq_beg, *gq_arc;
     int32_t *alive0, *alive1;
+    int32_t *near0, *near1;
     int32_t *seg0, *seg1;
     int32_t *deg;
 };
@@ -99,6 +100,8 @@ size_t carve(void *base, int64_t n, Carve *c)
     t.gq_arc = (int64_t *)take(sizeof(int64_t) * (nn + 1));
     t.alive0 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
+    t.near0 = (int32_t *)take(sizeof(int32_t) * nn);
+    t.near1 = (int32_t *)take(sizeof(int32_t) * nn);
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     t.seg1 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     // claim bits and working degrees adjacent: one L2 access-policy window
@@ -201,7 +204,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     int64_t *trace = opt ? opt->trace_out : nullptr;
     const int64_t trace_cap = (opt && opt->trace_out) ? opt->trace_cap : 0;
     const int bloom = (opt && (opt->flags & KCORE_FLAG_NO_BLOOM)) ? 0 : 1;
-    const int red = (opt && (opt->flags & KCORE_FLAG_NO_RED)) ? 0 : 1;
+    const int red = ((opt && (opt->flags & KCORE_FLAG_NO_RED)) ? 0 : 1) |
+                    ((opt && (opt->flags & KCORE_FLAG_NO_NEAR)) ? 0 : 2);
     const size_t smem = sizeof(Smem);
 
     const size_t need = carve(nullptr, n, nullptr);
@@ -234,6 +238,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.gq_arc = cv.gq_arc;
     A.alive[0] = cv.alive0;
     A.alive[1] = cv.alive1;
+    A.near[0] = cv.near0;
+    A.near[1] = cv.near1;
     A.seg_len[0] = cv.seg0;
     A.seg_len[1] = cv.seg1;
     A.nseg = grid;
@@ -245,7 +251,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
         KC_CUDA(cudaEventCreate(&ev0));
         KC_CUDA(cudaEventCreate(&ev1));
     }
-    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, red, trace,
+    k_init_state<<<1, 32, 0, st>>>(cv.S, n, solo, solo_scan, bloom, red, opt ? opt->near_min_alive : 0,
+                                   opt ? opt->near_window : 0, trace,
                                    trace ? opt->trace_cta_out : nullptr, trace_cap);
     KC_CUDA(cudaGetLastError());
     if (stats) KC_CUDA(cudaEventRecord(ev0, st));
@@ -333,6 +340,7 @@ launched:
         stats->solo_phases = c.st_solo;
         stats->barriers = c.st_bar;
         stats->scanned = c.st_scanned;
+        stats->near_scans = c.st_near;
         stats->arcs_walked = (int64_t)hS.arcs_walked;
         stats->compactions = c.st_compact;
         stats->hub_arcs = c.st_hubarcs;

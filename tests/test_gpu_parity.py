@@ -40,7 +40,11 @@ def _check(rp, ci, ref=None, **kw):
 
 
 VARIANTS = [dict(), dict(solo_arcs=16384, solo_scan=32768), dict(bloom=False), dict(algo=kc.ALGO_HOSTLOOP),
-            dict(solo_arcs=1 << 30, solo_scan=1 << 30)]
+            dict(solo_arcs=1 << 30, solo_scan=1 << 30),
+            # the near list forced on from the first level with tiny windows (every
+            # epoch boundary, theta crossing and level skip past theta is exercised)
+            dict(near_min_alive=1, near_window=1), dict(near_min_alive=1, near_window=3, red=False),
+            dict(near_min_alive=1, near_window=2, algo=kc.ALGO_HOSTLOOP), dict(near=False, red=False)]
 
 
 # ------------------------------------------------------------ paper pins
@@ -204,6 +208,25 @@ def _config_parity(name, check_cert=True):
     if check_cert:
         assert oracle.check_certificate(rp, ci, got, order.cpu().numpy()) == 0
     return st
+
+
+@pytest.mark.parametrize("cfg", ["C1", "chunglu-2^16", "rmat-s18"])
+@pytest.mark.parametrize("kw", [dict(near_min_alive=1, near_window=1), dict(near_min_alive=1, near_window=7),
+                                dict(near_min_alive=1, near_window=64), dict(near_min_alive=1 << 12, near_window=2),
+                                dict(near=False), dict(red=False, near_min_alive=1, near_window=5)])
+def test_near_list_windows(cfg, kw):
+    """Near-list epochs at every window size agree bit-exactly with the oracle
+    (DESIGN.md "near list"); stats count the near scans."""
+    spec = {"C1": kcgen.CONFIGS["C1"], "chunglu-2^16": kcgen.chunglu(1 << 16, 2.1, 1 << 20),
+            "rmat-s18": kcgen.rmat(18, 16)}[cfg]
+    rp, ci = kcgen.generate_host(spec)
+    ref = oracle.bz_core(rp, ci)
+    r, c = _to_dev(rp, ci)
+    core, st = kc.kcore_decompose(r, c, stats=True, **kw)
+    assert np.array_equal(core.cpu().numpy(), ref)
+    if kw.get("near", True) and kw.get("near_min_alive", 0) == 1:
+        assert st.near_scans > 0
+    assert st.levels == len(np.unique(ref))
 
 
 def test_config_C1():
