@@ -26,7 +26,7 @@ kcgen/libkcgen.so: kcgen/csrc/kcgen_host.c kcgen/csrc/kcgen_device.cu kcgen/csrc
 $(PKG)/lib/libkcore.so: $(KCORE_SRC)
 	mkdir -p $(PKG)/lib
 	$(NVCC) $(NVFLAGS) -Xptxas -v -Iinclude -I$(NCCL_DIR)/include -shared \
-	    $(PKG)/csrc/kcore.cu $(PKG)/csrc/kcore_mg.cu $(PKG)/csrc/kcore_extract.cu $(PKG)/csrc/kcore_mpm.cu $(PKG)/csrc/kcore_testhooks.cu -o $@ \
+	    $(PKG)/csrc/kcore.cu $(PKG)/csrc/kcore_mg.cu $(PKG)/csrc/kcore_extract.cu $(PKG)/csrc/kcore_mpm.cu $(PKG)/csrc/kcore_testhooks.cu $(PKG)/csrc/kcore_mgd.cu -o $@ \
 	    -L$(NCCL_DIR)/lib -l:libnccl.so.2 -Xlinker -rpath=$(NCCL_DIR)/lib 2> $(PKG)/lib/ptxas.log || (cat $(PKG)/lib/ptxas.log; false)
 
 clean:

@@ -238,14 +238,39 @@ int kcore_decompose_mg(const int64_t *rowptr_local, const int32_t *colidx_local,
                        int32_t *core_out_local, void *stream, void *nccl_comm,
                        kcore_stats *stats);
 
-/* The same protocol with `nranks` VIRTUAL ranks on the current device and a
- * device-memory loopback transport in place of NCCL (same kernels, same
- * driver, same routing).  Takes the GLOBAL CSR (DEVICE pointers), partitions
+/* The multi-GPU protocol with `nranks` VIRTUAL ranks (1..16) on the current
+ * device: the device-initiated kernel (KCORE_MG_DEVICE) with every rank's
+ * window a slice of one allocation; _ex with KCORE_MG_HOSTLOOP runs the
+ * host-driven protocol with a device-memory loopback transport instead of
+ * NCCL (same kernels, same driver, same routing).  Takes the GLOBAL CSR (DEVICE pointers), partitions
  * it into equal vertex ranges internally and writes the global core_out.  For
  * testing the multi-GPU protocol on one GPU.  Synchronises `stream`. */
 int kcore_decompose_mg_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n,
                                int64_t m, int32_t nranks, int32_t *core_out, void *stream,
                                kcore_stats *stats);
+
+/* Multi-GPU protocol selection (kcore_decompose_mg_ex / _virtual_ex):
+ *  KCORE_MG_DEVICE    device-initiated: ONE persistent
+ *                     kernel per rank; decrements and frontier appends go
+ *                     straight into the owner's memory (NCCL 2.28 symmetric
+ *                     windows over NVLink; slices of one allocation for
+ *                     virtual ranks); a device-side barrier per sub-round;
+ *                     no host round trip.  Default of kcore_decompose_mg_virtual.
+ *  KCORE_MG_HOSTLOOP  host-driven: grouped ncclSend/Recv of packed decrements
+ *                     and an all-reduce per sub-round.  Default of
+ *                     kcore_decompose_mg (the device path has not run on more
+ *                     than one GPU yet). */
+#define KCORE_MG_DEVICE 0
+#define KCORE_MG_HOSTLOOP 1
+
+int kcore_decompose_mg_ex(const int64_t *rowptr_local, const int32_t *colidx_local,
+                          int64_t n_global, int64_t v_begin, int64_t v_end, int64_t m_local,
+                          int32_t *core_out_local, void *stream, void *nccl_comm,
+                          int32_t mg_algo, kcore_stats *stats);
+
+int kcore_decompose_mg_virtual_ex(const int64_t *rowptr, const int32_t *colidx, int64_t n,
+                                  int64_t m, int32_t nranks, int32_t *core_out, void *stream,
+                                  int32_t mg_algo, kcore_stats *stats);
 
 /* NCCL plumbing for callers without their own communicator (the Python
  * binding uses these; the unique id is exchanged over torch.distributed).

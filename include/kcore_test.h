@@ -25,6 +25,12 @@ extern "C" {
 int kcore_test_ballot_compact(const int32_t *vid, const int32_t *pred, int32_t n, int32_t *prefix,
                               int32_t *buf, int32_t *e, void *stream);
 
+/* Phase trace of the next kcore_decompose_mg_virtual call (device-initiated
+ * protocol; development aid): DEVICE int64[cap][4] records {globaltimer ns,
+ * phase (-1 start, 0 init, 1 scan, 2 sub-round), k, removed so far} at every
+ * device barrier.  NULL disables. */
+int kcore_test_mgd_trace(int64_t *trace, int64_t cap);
+
 #ifdef __cplusplus
 }
 #endif

@@ -48,6 +48,7 @@ EXPORTS = (
     "kcore_validate_csr", "kcore_strerror", "kcore_version", "kcore_decompose_mg",
     "kcore_decompose_mg_virtual", "kcore_nccl_unique_id", "kcore_nccl_comm_init",
     "kcore_nccl_comm_destroy", "kcore_kshell", "kcore_kcore_mask", "kcore_kcore_subgraph", "kcore_mpm",
+    "kcore_decompose_mg_ex", "kcore_decompose_mg_virtual_ex",
 )
 
 
@@ -130,6 +131,8 @@ def _load():
         lib.kcore_version.restype = ctypes.c_char_p
         lib.kcore_decompose_mg.argtypes = [vp, vp, i64, i64, i64, i64, vp, vp, vp, ctypes.POINTER(_Stats)]
         lib.kcore_decompose_mg_virtual.argtypes = [vp, vp, i64, i64, i32, vp, vp, ctypes.POINTER(_Stats)]
+        lib.kcore_decompose_mg_ex.argtypes = [vp, vp, i64, i64, i64, i64, vp, vp, vp, i32, ctypes.POINTER(_Stats)]
+        lib.kcore_decompose_mg_virtual_ex.argtypes = [vp, vp, i64, i64, i32, vp, vp, i32, ctypes.POINTER(_Stats)]
         lib.kcore_nccl_unique_id.argtypes = [vp]
         lib.kcore_nccl_comm_init.argtypes = [ctypes.POINTER(vp), i32, vp, i32]
         lib.kcore_nccl_comm_destroy.argtypes = [vp]
@@ -252,8 +255,9 @@ def kcore_validate_csr(rowptr, colidx) -> int:
     return rc
 
 
-def kcore_decompose_mg_virtual(rowptr, colidx, nranks: int, *, stats: bool = False):
-    """Multi-GPU protocol with `nranks` virtual ranks on this GPU (global CSR in, global core out)."""
+def kcore_decompose_mg_virtual(rowptr, colidx, nranks: int, *, stats: bool = False, algo: int = 0):
+    """Multi-GPU protocol with `nranks` virtual ranks on this GPU (global CSR in, global core out).
+    algo 0 (KCORE_MG_DEVICE): the device-initiated kernel; 1 (KCORE_MG_HOSTLOOP): host-driven."""
     import torch
     _check_csr_tensors(rowptr, colidx)
     dev = rowptr.device
@@ -262,9 +266,9 @@ def kcore_decompose_mg_virtual(rowptr, colidx, nranks: int, *, stats: bool = Fal
     core = torch.empty(max(n, 0), dtype=torch.int32, device=dev)
     st = _Stats()
     with torch.cuda.device(dev):
-        rc = _load().kcore_decompose_mg_virtual(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
-                                                nranks, core.data_ptr() if n else None, _stream_ptr(dev),
-                                                ctypes.byref(st) if stats else None)
+        rc = _load().kcore_decompose_mg_virtual_ex(rowptr.data_ptr(), colidx.data_ptr() if m else None, n, m,
+                                                   nranks, core.data_ptr() if n else None, _stream_ptr(dev),
+                                                   int(algo), ctypes.byref(st) if stats else None)
     if rc != KCORE_OK:
         raise KcoreError(rc, "kcore_decompose_mg_virtual")
     return (core, Stats._from(st)) if stats else core

@@ -22,6 +22,7 @@
 // test the protocol on a single GPU).  Host-driven: two stream syncs per
 // sub-round (send counts, then the all-reduced control words).
 #include "kcore.h"
+#include "kcore_mgd.h"
 
 #include <climits>
 #include <cstdint>
@@ -545,9 +546,52 @@ extern "C" int kcore_nccl_comm_destroy(void *comm)
     return ncclCommDestroy((ncclComm_t)comm) == ncclSuccess ? KCORE_OK : KCORE_ENCCL;
 }
 
+static int mg_hostloop_nccl(const int64_t *rowptr_local, const int32_t *colidx_local, int64_t n_global,
+                            int64_t v_begin, int64_t v_end, int64_t m_local, int32_t *core_out_local,
+                            void *stream_, void *nccl_comm, kcore_stats *stats);
+static int mg_hostloop_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                               int32_t nranks, int32_t *core_out, void *stream_, kcore_stats *stats);
+
 extern "C" int kcore_decompose_mg(const int64_t *rowptr_local, const int32_t *colidx_local, int64_t n_global,
                                   int64_t v_begin, int64_t v_end, int64_t m_local, int32_t *core_out_local,
                                   void *stream_, void *nccl_comm, kcore_stats *stats)
+{
+    return mg_hostloop_nccl(rowptr_local, colidx_local, n_global, v_begin, v_end, m_local, core_out_local, stream_,
+                            nccl_comm, stats);
+}
+
+extern "C" int kcore_decompose_mg_ex(const int64_t *rowptr_local, const int32_t *colidx_local, int64_t n_global,
+                                     int64_t v_begin, int64_t v_end, int64_t m_local, int32_t *core_out_local,
+                                     void *stream_, void *nccl_comm, int32_t mg_algo, kcore_stats *stats)
+{
+    if (mg_algo == KCORE_MG_DEVICE)
+        return mgd_nccl(rowptr_local, colidx_local, n_global, v_begin, v_end, m_local, core_out_local, stream_,
+                        nccl_comm, stats);
+    if (mg_algo == KCORE_MG_HOSTLOOP)
+        return mg_hostloop_nccl(rowptr_local, colidx_local, n_global, v_begin, v_end, m_local, core_out_local,
+                                stream_, nccl_comm, stats);
+    return KCORE_EINVAL;
+}
+
+extern "C" int kcore_decompose_mg_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                                          int32_t nranks, int32_t *core_out, void *stream_, kcore_stats *stats)
+{
+    return mgd_virtual(rowptr, colidx, n, m, nranks, core_out, stream_, stats);
+}
+
+extern "C" int kcore_decompose_mg_virtual_ex(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                                             int32_t nranks, int32_t *core_out, void *stream_, int32_t mg_algo,
+                                             kcore_stats *stats)
+{
+    if (mg_algo == KCORE_MG_DEVICE) return mgd_virtual(rowptr, colidx, n, m, nranks, core_out, stream_, stats);
+    if (mg_algo == KCORE_MG_HOSTLOOP)
+        return mg_hostloop_virtual(rowptr, colidx, n, m, nranks, core_out, stream_, stats);
+    return KCORE_EINVAL;
+}
+
+static int mg_hostloop_nccl(const int64_t *rowptr_local, const int32_t *colidx_local, int64_t n_global,
+                            int64_t v_begin, int64_t v_end, int64_t m_local, int32_t *core_out_local,
+                            void *stream_, void *nccl_comm, kcore_stats *stats)
 {
     if (!nccl_comm || n_global < 0 || n_global >= ((int64_t)1 << 31) || v_begin < 0 || v_end < v_begin ||
         v_end > n_global || m_local < 0)
@@ -596,8 +640,8 @@ extern "C" int kcore_decompose_mg(const int64_t *rowptr_local, const int32_t *co
     return rc;
 }
 
-extern "C" int kcore_decompose_mg_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
-                                          int32_t nranks, int32_t *core_out, void *stream_, kcore_stats *stats)
+static int mg_hostloop_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t m,
+                               int32_t nranks, int32_t *core_out, void *stream_, kcore_stats *stats)
 {
     if (n < 0 || n >= ((int64_t)1 << 31) || m < 0 || nranks < 1 || nranks > kMaxRanks) return KCORE_EINVAL;
     if (n > 0 && (!rowptr || !core_out)) return KCORE_EINVAL;

@@ -98,10 +98,15 @@ class NcclComm:
             pass
 
 
+MG_DEVICE = 0    # device-initiated persistent kernel over NCCL symmetric windows
+MG_HOSTLOOP = 1  # host-driven NCCL exchange per sub-round (default of kcore_decompose_mg)
+
+
 def kcore_decompose_mg(rowptr_local, colidx_local, n_global: int, v_begin: int, v_end: int,
-                       comm: NcclComm, *, stats: bool = False):
+                       comm: NcclComm, *, stats: bool = False, algo: int = MG_HOSTLOOP):
     """This rank's core numbers (int32 CUDA tensor of v_end-v_begin entries).
-    Collective over `comm`; synchronises the current stream per sub-round."""
+    Collective over `comm`.  algo=MG_HOSTLOOP synchronises the stream per
+    sub-round; algo=MG_DEVICE runs one persistent kernel per rank."""
     import torch
     from . import KcoreError, Stats, _Stats, _check_csr_tensors, _load, _stream_ptr
     _check_csr_tensors(rowptr_local, colidx_local)
@@ -113,10 +118,10 @@ def kcore_decompose_mg(rowptr_local, colidx_local, n_global: int, v_begin: int, 
     st = _Stats()
     m_local = colidx_local.numel()
     with torch.cuda.device(dev):
-        rc = _load().kcore_decompose_mg(rowptr_local.data_ptr(), colidx_local.data_ptr() if m_local else None,
-                                        n_global, v_begin, v_end, m_local,
-                                        core.data_ptr() if nl else None, _stream_ptr(dev), comm.handle,
-                                        ctypes.byref(st) if stats else None)
+        rc = _load().kcore_decompose_mg_ex(rowptr_local.data_ptr(), colidx_local.data_ptr() if m_local else None,
+                                           n_global, v_begin, v_end, m_local,
+                                           core.data_ptr() if nl else None, _stream_ptr(dev), comm.handle,
+                                           int(algo), ctypes.byref(st) if stats else None)
     if rc != KCORE_OK:
         raise KcoreError(rc, "kcore_decompose_mg")
     return (core, Stats._from(st)) if stats else core

@@ -33,25 +33,49 @@ GRAPHS = [
 ]
 
 
+GRAPHS += [
+    ("star_big_hub", lambda: kcgen.csr_from_edges(20001, [(0, i) for i in range(1, 20001)])),
+    ("bowtie_fan", lambda: kcgen.csr_from_edges(
+        6001, [e for i in range(3000) for e in ((0, 1 + 2 * i), (0, 2 + 2 * i), (1 + 2 * i, 2 + 2 * i))])),
+]
+
+
 @pytest.mark.parametrize("name,make", GRAPHS)
-@pytest.mark.parametrize("P", [1, 2, 3, 4, 8])
-def test_virtual_ranks_match_oracle(name, make, P):
+@pytest.mark.parametrize("P", [1, 2, 3, 4, 5, 8])
+@pytest.mark.parametrize("algo", [0, 1])
+def test_virtual_ranks_match_oracle(name, make, P, algo):
+    """Both protocols (0: device-initiated, 1: host-driven) with P virtual ranks."""
     rp, ci = make()
     ref = oracle.bz_core(rp, ci)
     r, c = _dev(rp, ci)
-    got, st = kc.kcore_decompose_mg_virtual(r, c, P, stats=True)
-    assert np.array_equal(got.cpu().numpy(), ref), (name, P)
+    got, st = kc.kcore_decompose_mg_virtual(r, c, P, stats=True, algo=algo)
+    assert np.array_equal(got.cpu().numpy(), ref), (name, P, algo)
     if ref.size and ref.max() > 0:
         assert st.kmax == ref.max()
+        assert st.levels == len(np.unique(ref))
 
 
-def test_virtual_ranks_config_C1():
-    rp, ci = kcgen.generate_host(kcgen.CONFIGS["C1"])
+@pytest.mark.parametrize("cfg", ["C1", "C2", "C3"])
+def test_virtual_ranks_configs(cfg):
+    """Device-initiated protocol, P = 2..8 virtual ranks, full-size C1-C3."""
+    rp, ci = kcgen.generate_host(kcgen.CONFIGS[cfg]) if cfg == "C1" else (None, None)
+    if cfg != "C1":
+        r, c = kcgen.generate_device(kcgen.CONFIGS[cfg])
+        rp, ci = r.cpu().numpy(), c.cpu().numpy()
     ref = oracle.bz_core(rp, ci)
     r, c = _dev(rp, ci)
-    for P in (2, 8):
+    for P in ((2, 3, 4, 5, 6, 7, 8) if cfg == "C1" else (2, 8)):
         got = kc.kcore_decompose_mg_virtual(r, c, P)
-        assert np.array_equal(got.cpu().numpy(), ref), P
+        assert np.array_equal(got.cpu().numpy(), ref), (cfg, P)
+
+
+@pytest.mark.slow
+def test_virtual_ranks_config_C4():
+    r, c = kcgen.generate_device(kcgen.CONFIGS["C4"])
+    ref = kc.kcore_decompose(r, c)  # itself pinned to the oracle by test_config_C4_full_size
+    for P in (2, 4, 8):
+        got = kc.kcore_decompose_mg_virtual(r, c, P)
+        assert torch.equal(got, ref), P
 
 
 def _free_port():
@@ -75,6 +99,10 @@ def test_nccl_transport_single_rank():
         r, c = _dev(lrp, lci)
         got = kc.kcore_decompose_mg(r, c, n, vb, ve, comm)
         assert np.array_equal(got.cpu().numpy(), ref)
+        # the device-initiated protocol through NCCL symmetric memory (one rank:
+        # window registration, peer pointers from ncclGetPeerPointer, device barrier)
+        got2 = kc.kcore_decompose_mg(r, c, n, vb, ve, comm, algo=parallel.MG_DEVICE)
+        assert np.array_equal(got2.cpu().numpy(), ref)
         comm.close()
     finally:
         dist.destroy_process_group()
