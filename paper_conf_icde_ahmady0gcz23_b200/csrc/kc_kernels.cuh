@@ -163,6 +163,15 @@ constexpr int kTraceFields = 8;
 #ifndef KC_NEAR_W
 #define KC_NEAR_W 16
 #endif
+#ifndef KC_BLOOM_GATE
+#define KC_BLOOM_GATE 1  // build the alive-set filter only when the CTA walks >= 1/KC_BLOOM_GATE of the list's length
+#endif
+#ifndef KC_SCAN_EC
+#define KC_SCAN_EC 0  // 1 (ablation): level-scan compaction with block scans (Fig. 9) instead of warp ballots
+#endif
+#ifndef KC_NO_SMBUF
+#define KC_NO_SMBUF 0  // 1 (ablation): no shared-memory frontier -- every claimed vertex goes to the global queue
+#endif
 #ifndef KC_NEAR
 #define KC_NEAR 1  // 0: compile the near list out (walks never test for theta crossings)
 #endif
@@ -528,7 +537,7 @@ __device__ __noinline__ void route_won(const KArgs &A, Smem &sm, int wib, bool w
             atomicAdd(&sm.removed, __popc(b));
         }
     }
-    const bool cand = won && dv > 0 && dv <= sm.bud_hub && nx >= 0;  // nx < 0: no local list
+    const bool cand = !KC_NO_SMBUF && won && dv > 0 && dv <= sm.bud_hub && nx >= 0;  // nx < 0: no local list
     const unsigned bc = __ballot_sync(kFull, cand);
     bool wantl = false;
     int lbase = 0;
@@ -616,7 +625,7 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
     unsigned cm = 0;
 #pragma unroll
     for (int r = 0; r < 4; r++)
-        if (((wm >> r) & 1u) && dd[r] > 0 && dd[r] <= sm.bud_hub && nx >= 0) cm |= 1u << r;
+        if (!KC_NO_SMBUF && ((wm >> r) & 1u) && dd[r] > 0 && dd[r] <= sm.bud_hub && nx >= 0) cm |= 1u << r;
     unsigned cb[4];
     int coff[4], ctot = 0, sumd = 0;
 #pragma unroll
@@ -1199,11 +1208,13 @@ __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
 // cascade walked by one CTA.
 __device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &sm, int64_t arcs)
 {
-    (void)arcs;
     if (!A.S->prm.bloom) return false;
     const bool have = sm.bloom_on != 0;
     if (have && c.src_len * 2 > sm.bloom_level) return true;
     if (c.src_sel < 0 || c.src_len > kBloomMaxA) return have;
+    // building costs one pass over the alive list per CTA: only for a walk
+    // of comparable size (CTA-uniform: arcs is this CTA's pending walk)
+    if (KC_BLOOM_GATE > 0 && arcs * KC_BLOOM_GATE < c.src_len) return have;
     bloom_build(A, c, sm);
     return true;
 }
@@ -1279,7 +1290,13 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
         }
     };
     load_chunk(lo + (int64_t)wib * CH);
+#if KC_SCAN_EC
+    // (ablation: block-level compaction needs every warp in every step)
+    for (int64_t base = lo; base < hi; base += (int64_t)kWarps * CH) {
+        const int64_t off = base + (int64_t)wib * CH;
+#else
     for (int64_t off = lo + (int64_t)wib * CH; off < hi; off += (int64_t)kWarps * CH) {
+#endif
         int32_t vv[kScanItems], dd[kScanItems];
         if (!KC_SCAN_PIPE && off != lo + (int64_t)wib * CH) load_chunk(off);
 #pragma unroll
@@ -1322,7 +1339,20 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
                     if ((nm >> j) & 1u) ndst[pos++] = vv[j];
             }
         }
+#if KC_SCAN_EC
+        if (dst) {  // the paper's block-level compaction (Fig. 9): two-stage block scan
+            const unsigned long long ex = block_excl_scan(sm, (unsigned long long)__popc(km));
+            int pos = sm.kcur + (int)ex;
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++)
+                if ((km >> j) & 1u) dst[pos++] = vv[j];
+            __syncthreads();
+            if (threadIdx.x == 0) sm.kcur += (int)sm.tot_q;
+        }
+        if (false) {
+#else
         if (dst) {
+#endif
             int mine = __popc(km), incl = mine;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {

@@ -345,3 +345,25 @@ def test_concurrent_calls_on_two_streams():
             s.synchronize()
         for o, ref in zip(outs, refs):
             assert np.array_equal(o.cpu().numpy(), ref), rep
+
+
+@pytest.mark.slow
+def test_config_C5_one_gpu():
+    """C5 (R-MAT s27 ef32, 8.36 G arcs > 2^31, BASELINE.json configs[4]) on ONE
+    B200: generated on the device in owner-range chunks, decomposed, then
+    compared element by element with the serial oracle on the host (needs
+    ~45 GB of host RAM; the I2 + I4 certificate of the device's peel order is
+    checked by tools/c5_run.py, profiles/r2/c5_r2.json)."""
+    import psutil
+    if psutil.virtual_memory().available < (60 << 30) or torch.cuda.get_device_properties(0).total_memory < (100 << 30):
+        pytest.skip("C5 needs ~60 GB host RAM and ~60 GB device memory")
+    r, c = kcgen.generate_device_chunked(kcgen.CONFIGS["C5"], chunks=8)
+    n = r.numel() - 1
+    core, st = kc.kcore_decompose(r, c, stats=True)
+    assert st.arcs_walked <= c.numel() and st.levels > 500
+    rp, ci = r.cpu().numpy(), c.cpu().numpy()
+    del r, c
+    torch.cuda.empty_cache()
+    got = core.cpu().numpy()
+    ref = oracle.bz_core(rp, ci)
+    assert np.array_equal(got, ref)

@@ -9,7 +9,7 @@ build() {
   tag=$1; shift
   /usr/local/cuda/bin/nvcc -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 -Xcompiler -fPIC \
     --expt-relaxed-constexpr -Iinclude -I$NCCL_DIR/include -shared "$@" \
-    paper_conf_icde_ahmady0gcz23_b200/csrc/kcore.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_mg.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_extract.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_mpm.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_testhooks.cu \
+    paper_conf_icde_ahmady0gcz23_b200/csrc/kcore.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_mg.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_extract.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_mpm.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_testhooks.cu paper_conf_icde_ahmady0gcz23_b200/csrc/kcore_mgd.cu \
     -o $OUT/$tag.so -L$NCCL_DIR/lib -l:libnccl.so.2 -Xlinker -rpath=$NCCL_DIR/lib
   echo built $tag
 }
