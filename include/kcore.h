@@ -69,9 +69,12 @@ typedef enum {
 #define KCORE_FLAG_NO_L2_PERSIST 2 /* do not pin the working degrees in L2 (ablation).  By    */
                                 /* default the call launches with a persisting L2 access- */
                                 /* policy window over its claim bits + working degrees,   */
-                                /* raising cudaLimitPersistingL2CacheSize (device-wide,   */
-                                /* never lowered) to the window size if it is smaller, and */
-                                /* returns the lines to normal priority after the kernel. */
+                                /* raising cudaLimitPersistingL2CacheSize (device-wide)   */
+                                /* to the window size if it is smaller, and returns the   */
+                                /* lines to normal priority after the kernel.  A call that */
+                                /* synchronises (stats != NULL, kcore_decompose_host)     */
+                                /* restores the previous limit before returning; an       */
+                                /* asynchronous call leaves it raised.                    */
 #define KCORE_FLAG_NO_RED 4     /* ablation: heavy HUB phases keep returning atomicSub     */
                                 /* (default: phases walking >= 2^21 arcs over an alive set */
                                 /* <= 1/8 of them use non-returning red.global.add and a   */

@@ -217,6 +217,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     int64_t hl_launches = 0;
     const char *l2_base = nullptr;
     State hS;
+    size_t prev_limit = 0;
+    bool limit_raised = false;
     Carve cv;
     KArgs A;
     if (opt && opt->workspace) {
@@ -278,6 +280,8 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
             cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize);
             const size_t want = std::min(wbytes, (size_t)di.persist_max);
             if (lim < want) {
+                prev_limit = lim;
+                limit_raised = true;
                 KC_CUDA(cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want));
                 KC_CUDA(cudaDeviceGetLimit(&lim, cudaLimitPersistingL2CacheSize));
             }
@@ -332,6 +336,11 @@ launched:
     if (stats) {
         KC_CUDA(cudaMemcpyAsync(&hS, cv.S, sizeof(State), cudaMemcpyDeviceToHost, st));
         KC_CUDA(cudaStreamSynchronize(st));
+        // the call has completed: hand the L2 set-aside back (a stream-ordered
+        // restore does not exist; asynchronous calls leave the raised limit --
+        // include/kcore.h, KCORE_FLAG_NO_L2_PERSIST)
+        if (limit_raised) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, prev_limit);
+        limit_raised = false;
         float ms = 0.f;
         cudaEventElapsedTime(&ms, ev0, ev1);
         const Ctrl &c = hS.pub;
@@ -407,7 +416,10 @@ extern "C" int kcore_decompose_host(const int64_t *rowptr_h, const int32_t *coli
     KC_CUDA(cudaMemcpyAsync(d_rp, rowptr_h, sizeof(int64_t) * (size_t)(n + 1), cudaMemcpyHostToDevice, st));
     if (m > 0)
         KC_CUDA(cudaMemcpyAsync(d_ci, colidx_h, sizeof(int32_t) * (size_t)m, cudaMemcpyHostToDevice, st));
-    rc = kcore_decompose_ex(d_rp, d_ci, n, m, d_core, st, opt, stats);
+    {
+        kcore_stats local;  // the host path synchronises anyway: stats make the call restore the L2 limit
+        rc = kcore_decompose_ex(d_rp, d_ci, n, m, d_core, st, opt, stats ? stats : &local);
+    }
     if (rc) goto done;
     KC_CUDA(cudaMemcpyAsync(core_h, d_core, sizeof(int32_t) * (size_t)n, cudaMemcpyDeviceToHost, st));
     KC_CUDA(cudaStreamSynchronize(st));

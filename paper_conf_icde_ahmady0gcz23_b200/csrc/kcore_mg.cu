@@ -290,10 +290,11 @@ struct NcclTransport : Transport {
     cudaStream_t st;
     unsigned long long *d_cnt = nullptr;  // [2][P]
     int32_t *d_red = nullptr;
+    bool ok = false;  // both scratch buffers allocated
     NcclTransport(ncclComm_t c, int p, int r, cudaStream_t s) : comm(c), P(p), rank(r), st(s)
     {
-        cudaMallocAsync((void **)&d_cnt, sizeof(unsigned long long) * 2 * P, st);
-        cudaMallocAsync((void **)&d_red, sizeof(int32_t) * 2, st);
+        ok = cudaMallocAsync((void **)&d_cnt, sizeof(unsigned long long) * 2 * P, st) == cudaSuccess &&
+             cudaMallocAsync((void **)&d_red, sizeof(int32_t) * 2, st) == cudaSuccess;
     }
     ~NcclTransport()
     {
@@ -605,7 +606,10 @@ static int mg_hostloop_nccl(const int64_t *rowptr_local, const int32_t *colidx_l
     if (ncclCommCount(comm, &P) != ncclSuccess || ncclCommUserRank(comm, &rank) != ncclSuccess) return KCORE_ENCCL;
     if (P > kMaxRanks) return KCORE_EUNSUPPORTED;
     NcclTransport T(comm, P, rank, st);
-    // owner table: every rank contributes its v_begin (ranges tile [0, n) in rank order)
+    // owner table: every rank contributes its v_begin (ranges tile [0, n) in rank order).
+    // The validity of every rank's range (and of its scratch) is all-reduced, so
+    // all ranks return the same status together -- none is left waiting in a
+    // collective of the protocol.
     Owners O;
     memset(&O, 0, sizeof(O));
     O.nranks = P;
@@ -618,9 +622,11 @@ static int mg_hostloop_nccl(const int64_t *rowptr_local, const int32_t *colidx_l
         MG_CK(cudaFreeAsync(d_vb, st));
         MG_CK(cudaStreamSynchronize(st));
         O.start[P] = n_global;
-        if (O.start[rank] != v_begin || (rank + 1 < P && O.start[rank + 1] != v_end) ||
-            (rank + 1 == P && v_end != n_global) || O.start[0] != 0)
-            return KCORE_EINVAL;
+        const bool mine_ok = T.ok && O.start[rank] == v_begin && (rank + 1 >= P || O.start[rank + 1] == v_end) &&
+                             (rank + 1 != P || v_end == n_global) && O.start[0] == 0;
+        int32_t flag[2] = {mine_ok ? 0 : -1, INT_MAX};
+        MG_RC(T.allreduce_min2(flag));  // min over ranks: -1 if any rank is invalid
+        if (flag[0] < 0) return T.ok ? KCORE_EINVAL : KCORE_ENOMEM;
     }
     std::vector<RankView> R(1);
     RankView &v = R[0];
