@@ -145,7 +145,7 @@ constexpr int kTraceFields = 8;
 #define KC_RED_MIN (1 << 21)
 #endif
 #ifndef KC_RED_RATIO
-#define KC_RED_RATIO 8
+#define KC_RED_RATIO 4
 #endif
 #ifndef KC_RED_UNROLL
 #define KC_RED_UNROLL 8
@@ -1270,6 +1270,7 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
 // deg == k -> claim + route (local frontier or global queue); deg > k ->
 // min for the level skip and, when compacting, ballot compaction (Fig. 8(c))
 // into dst[0..) with a shared-memory cursor.  No block sync, no global atomics.
+template <bool IDENT>
 __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_t *src, int64_t lo,
                            int64_t hi, int32_t *dst, int &lmin, int &gcnt, int32_t *ndst = nullptr,
                            unsigned long long *ntail = nullptr)
@@ -1314,8 +1315,23 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
             // in a lazily compacted list fail the claim.  At k = 0 the frontier
             // is the isolated vertices: nothing walks, nothing races.
             if (vv[j] < 0) continue;
-            if (dd[j] <= k) { if (k == 0 || claim(A, vv[j])) wm |= 1u << j; }
+            if (dd[j] <= k) { if (IDENT || k == 0 || claim(A, vv[j])) wm |= 1u << j; }
             else if (dd[j] > k) { lmin = min(lmin, dd[j]); km |= 1u << j; }
+        }
+        if (IDENT && k > 0) {
+            // identity scan (ids lo..hi-1, the first level): the 32 lanes of item j
+            // hold 32 consecutive ids starting at a multiple of 32 (lo is aligned),
+            // i.e. ONE claim-bit word -- one atomicOr for the warp instead of 32
+            // serialised ones on the same address
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++) {
+                const unsigned bits = __ballot_sync(kFull, (wm >> j) & 1u);
+                if (!bits) continue;
+                uint32_t old = 0u;
+                if (lane == 0) old = atom_or_claim(A.claimed + ((uint32_t)(vv[j] - lane) >> 5), bits, pol);
+                old = __shfl_sync(kFull, old, 0);
+                if ((old >> lane) & 1u) wm &= ~(1u << j);
+            }
         }
         if (ndst) {  // near list: k < deg <= theta (a near scan's compaction, or a build)
             unsigned nm = 0;
@@ -1413,7 +1429,7 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
     if (c.near_scan) {  // the near list: one contiguous run, an even slice per CTA, no alive compaction
         const int64_t L = c.near_len;
         const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
-        scan_range(A, c, sm, A.near[c.near_cur], lo, hi, nullptr, lmin, gcnt, ndst, ntail);
+        scan_range<false>(A, c, sm, A.near[c.near_cur], lo, hi, nullptr, lmin, gcnt, ndst, ntail);
         __syncthreads();
         return;
     }
@@ -1426,16 +1442,22 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
     if (c.src_sel < 0 || c.src_single) {
         // contiguous source of c.src_len entries: an even slice per CTA
         const int64_t L = c.src_len;
-        const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
-        scan_range(A, c, sm, srcb, lo, hi, dst, lmin, gcnt, ndst, ntail);
+        if (c.src_sel < 0) {  // the identity: 32-aligned slices (one claim-bit word per warp item)
+            const int64_t W = (L + 31) / 32;
+            const int64_t lo = solo ? 0 : 32 * ((W * bid) / nblk), hi = solo ? L : min(L, 32 * ((W * (bid + 1)) / nblk));
+            scan_range<true>(A, c, sm, nullptr, lo, hi, dst, lmin, gcnt, ndst, ntail);
+        } else {
+            const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
+            scan_range<false>(A, c, sm, srcb, lo, hi, dst, lmin, gcnt, ndst, ntail);
+        }
     } else if (!solo) {
         // this CTA wrote its own segment's length at the last compaction
         const int64_t len = sm.seg_cache_ok[c.src_sel] ? sm.seg_cache[c.src_sel] : ld_cg_i32(A.seg_len[c.src_sel] + bid);
-        scan_range(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
+        scan_range<false>(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
     } else {
         for (int b = 0; b < A.nseg; b++) {
             const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
-            if (len) scan_range(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
+            if (len) scan_range<false>(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
         }
     }
     __syncthreads();

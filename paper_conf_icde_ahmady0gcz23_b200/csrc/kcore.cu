@@ -98,8 +98,9 @@ size_t carve(void *base, int64_t n, Carve *c)
     t.gq_v = (int32_t *)take(sizeof(int32_t) * nn);
     t.gq_beg = (int64_t *)take(sizeof(int64_t) * nn);
     t.gq_arc = (int64_t *)take(sizeof(int64_t) * (nn + 1));
-    t.alive0 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
-    t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + kMaxSeg));
+    // segments of ceil(n/grid) + 32 entries (the identity scan's slices are 32-aligned)
+    t.alive0 = (int32_t *)take(sizeof(int32_t) * (nn + 33 * (size_t)kMaxSeg));
+    t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + 33 * (size_t)kMaxSeg));
     t.near0 = (int32_t *)take(sizeof(int32_t) * nn);
     t.near1 = (int32_t *)take(sizeof(int32_t) * nn);
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
@@ -245,7 +246,7 @@ extern "C" int kcore_decompose_ex(const int64_t *rowptr, const int32_t *colidx, 
     A.seg_len[0] = cv.seg0;
     A.seg_len[1] = cv.seg1;
     A.nseg = grid;
-    A.seg_R = (n + A.nseg - 1) / A.nseg;
+    A.seg_R = (n + A.nseg - 1) / A.nseg + 32;  // room for a 32-aligned identity slice
     A.S = cv.S;
     A.n = n;
 
