@@ -241,8 +241,10 @@ def run_gpu(args):
         dist.all_reduce(t)
         m_arcs = int(t.item())
 
+        algo = parallel.MG_DEVICE if args.mg_algo == "device" else parallel.MG_HOSTLOOP
+
         def step():
-            return kc.kcore_decompose_mg(rowptr, colidx, n, vb, ve, comm, stats=True)
+            return kc.kcore_decompose_mg(rowptr, colidx, n, vb, ve, comm, stats=True, algo=algo)
     m_und = m_arcs // 2
     torch.cuda.synchronize()
 
@@ -367,6 +369,20 @@ def run_gpu(args):
                            "ms_per_step": statistics.mean(mm), "iterations": it_m,
                            "arcs_gathered": st_m.arcs_walked, "equals_peel": bool(torch.equal(a_m, core))}
         del a_m
+    if world == 1 and not args.force_mg and not args.no_mpm:
+        # the multi-GPU protocol (device-initiated) with 8 virtual ranks on
+        # this one GPU, same graph: context for the 8-GPU design, not a scaling number
+        torch.cuda.empty_cache()
+        mv = []
+        for rep_ in range(4):
+            flush.fill_(1)
+            c_mg, st_mg = kc.kcore_decompose_mg_virtual(rowptr, colidx, 8, stats=True)
+            if rep_:
+                mv.append(st_mg.kernel_ms)
+        line["alt_mg_virtual8"] = {"value": m_und / (statistics.median(mv) * 1e-3) / 1e6, "unit": "Medges/s",
+                                   "ms_per_step": statistics.median(mv), "sub_rounds": st_mg.phases,
+                                   "device_barriers": st_mg.barriers, "equals_peel": bool(torch.equal(c_mg, core))}
+        del c_mg
     if world == 1 and not args.force_mg and not args.no_configs:
         # the other single-GPU configs (BASELINE.json configs[0..2]) with the same protocol
         line["per_config"] = per_config(args, kc, kcgen, flush, stream, peak,
@@ -406,6 +422,8 @@ def main():
     ap.add_argument("--no-mpm", action="store_true", help="skip the MPM context measurement")
     ap.add_argument("--force-mg", action="store_true", help="run the multi-GPU path even at N=1")
     ap.add_argument("--no-configs", action="store_true", help="skip the C1-C3 per-config measurements")
+    ap.add_argument("--mg-algo", default="host", choices=["host", "device"],
+                    help="N > 1: host-driven NCCL exchange (default) or the device-initiated kernel")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
