@@ -64,6 +64,9 @@ constexpr int kWarps = kBlk / 32;
 constexpr int32_t kRemoved = 1 << 30;  // added to deg when a vertex is removed
 constexpr int32_t kDead = 1 << 29;     // deg >= kDead: removed
 constexpr int kChunk = 256;            // chunk queue granularity (arcs)
+static_assert(kChunk <= 256, "chunk length - 1 is stored in 8 bits");
+constexpr int kNearW = 16;             // near window W (DESIGN R15): levels k..k+W scan only the near list
+constexpr int64_t kNearMin = 1 << 17;  // alive vertices (all ranks) from which a FULL scan builds one
 constexpr int kSmall = 64;             // longer rows are walked through the chunk queue
 constexpr unsigned kFull = 0xffffffffu;
 
@@ -87,8 +90,7 @@ struct RankLocal {
     int32_t *alive[2];     // per-CTA segments [G][seg_cap] of owned local ids
     int32_t *seglen[2];    // [G]
     int64_t seg_cap;
-    int64_t *chunk_beg;    // big-row chunks of the current sub-round
-    uint32_t *chunk_tag;   // (sub-round epoch << 12) | (len - 1), written last
+    unsigned long long *chunk;  // long-row chunks: (epoch << 44) | ((len-1) << 36) | begin, one atomic word
     int64_t chunk_cap;
     unsigned long long *lctl;  // rank-local cursors: [0] item pop [1] items done [2] chunk tail [3] chunk pop
     int64_t nl;
@@ -106,6 +108,7 @@ struct Args {
     char *peer[kMaxR];  // window base of every rank (virtual; NCCL: peer_dev)
     char *const *peer_dev;
     int64_t off_tail, off_deg, off_in0, off_in1, in_cap;
+    int64_t off_near0, off_near1;  // near lists [2][nl_max] (their tails follow the inbox tails)
     int64_t *stats;     // [0] levels [1] sub-rounds [2] barriers [3] kmax [4] arcs
     int64_t *trace;     // optional [trace_cap][8]: {globaltimer, phase (0 init 1 scan 2 peel), k, pushed,
                         //  block 0's peel: items done, chunks done, end}
@@ -121,6 +124,8 @@ struct Smem {
     unsigned long long snap_pushed, snap_prev;
     int snap_min, snap_par;
     float inv_n;  // P / n
+    int th1;      // theta + 1 of the running near epoch (INT_MIN: none): walks append theta+1 -> theta crossings
+    int near_cur; // near[near_cur] is the list the next near scan reads (and walks append to)
 };
 
 // ------------------------------------------------------------ scoped atomics
@@ -168,6 +173,14 @@ __device__ __forceinline__ unsigned long long *tail_of(const Args &A, const Smem
 {
     return (unsigned long long *)(sm.peer[r] + A.off_tail) + which;
 }
+__device__ __forceinline__ int32_t *near_of(const Args &A, const Smem &sm, int r, int which)
+{
+    return (int32_t *)(sm.peer[r] + (which ? A.off_near1 : A.off_near0));
+}
+__device__ __forceinline__ unsigned long long *ntail_of(const Args &A, const Smem &sm, int r, int which)
+{
+    return (unsigned long long *)(sm.peer[r] + A.off_tail) + 2 + which;
+}
 
 // Device barrier over every CTA of every rank, two-level: the CTAs of a rank
 // arrive on a rank-local counter; the rank's last arriver resets the rank's
@@ -182,7 +195,7 @@ enum : int { L_POP = 0, L_DONE = 1, L_CTAIL = 2, L_CPOP = 3, L_BAR = 4, L_GEN = 
 
 // Virtual ranks (one launch holds every rank): a single-level barrier over all
 // P*G CTAs; the last arriver resets every rank's cursors itself.
-__device__ void gbar_flat(const Args &A, Smem &sm, int reset_par, int mode)
+__device__ void gbar_flat(const Args &A, Smem &sm, int reset_par, int mode, int near_reset)
 {
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -203,6 +216,7 @@ __device__ void gbar_flat(const Args &A, Smem &sm, int reset_par, int mode)
                 unsigned long long *lc = A.R[r].lctl;
                 lc[L_POP] = lc[L_DONE] = lc[L_CTAIL] = lc[L_CPOP] = 0ULL;
                 if (reset_par >= 0) *tail_of(A, sm, A.rank0 + r, reset_par) = 0ULL;
+                if (near_reset >= 0) *ntail_of(A, sm, A.rank0 + r, near_reset) = 0ULL;
             }
             c->bar_count = 0u;
             __threadfence();
@@ -219,10 +233,10 @@ __device__ void gbar_flat(const Args &A, Smem &sm, int reset_par, int mode)
     __syncthreads();
 }
 
-__device__ void gbar(const Args &A, Smem &sm, int rl, int reset_par, int mode)
+__device__ void gbar(const Args &A, Smem &sm, int rl, int reset_par, int mode, int near_reset = -1)
 {
     if (A.PL == A.P) {
-        gbar_flat(A, sm, reset_par, mode);
+        gbar_flat(A, sm, reset_par, mode, near_reset);
         return;
     }
     __syncthreads();
@@ -237,6 +251,7 @@ __device__ void gbar(const Args &A, Smem &sm, int rl, int reset_par, int mode)
             lc[L_BAR] = 0ULL;
             lc[L_POP] = lc[L_DONE] = lc[L_CTAIL] = lc[L_CPOP] = 0ULL;
             if (reset_par >= 0) *tail_of(A, sm, A.rank0 + rl, reset_par) = 0ULL;
+            if (near_reset >= 0) *ntail_of(A, sm, A.rank0 + rl, near_reset) = 0ULL;
             Ctl *c = gctl(sm);
             const unsigned gen = ld_volatile_u32(&c->bar_gen);
             fence(sys);
@@ -324,7 +339,10 @@ __device__ void phase_init(const Args &A, Smem &sm, int rl, int b)
 }
 
 // ---------------------------------------------------------------- SCAN (Alg. 2)
-__device__ void phase_scan(const Args &A, Smem &sm, int rl, int b, int k, int sel, int par)
+// mode 0: FULL scan of the alive segments; 1: FULL scan that also builds the
+// next near list (k < deg <= theta into near[near_cur ^ 1]); 2: near scan (the
+// rank's near[near_cur] split over its CTAs, survivors into near[near_cur ^ 1]).
+__device__ void phase_scan(const Args &A, Smem &sm, int rl, int b, int k, int sel, int par, int mode, int theta)
 {
     const RankLocal &R = A.R[rl];
     const int me = A.rank0 + rl;
@@ -332,20 +350,42 @@ __device__ void phase_scan(const Args &A, Smem &sm, int rl, int b, int k, int se
     int32_t *deg = deg_of(A, sm, me);
     int32_t *inbox = inbox_of(A, sm, me, par);
     unsigned long long *tail = tail_of(A, sm, me, par);
-    const int32_t *src = R.alive[sel] + (int64_t)b * R.seg_cap;
-    int32_t *dst = R.alive[sel ^ 1] + (int64_t)b * R.seg_cap;
-    const int len = R.seglen[sel][b];
+    const int32_t *src;
+    int32_t *dst = nullptr;
+    int64_t lo = 0, hi;
+    if (mode == 2) {
+        const int64_t L = (int64_t)*(volatile unsigned long long *)ntail_of(A, sm, me, sm.near_cur);
+        src = near_of(A, sm, me, sm.near_cur);
+        lo = L * b / A.G;
+        hi = L * (b + 1) / A.G;
+    } else {
+        src = R.alive[sel] + (int64_t)b * R.seg_cap;
+        dst = R.alive[sel ^ 1] + (int64_t)b * R.seg_cap;
+        hi = R.seglen[sel][b];
+    }
+    int32_t *ndst = mode ? near_of(A, sm, me, sm.near_cur ^ 1) : nullptr;
+    unsigned long long *ntail = mode ? ntail_of(A, sm, me, sm.near_cur ^ 1) : nullptr;
     if (threadIdx.x == 0) sm.kcur = 0;
     __syncthreads();
     int lmin = INT_MAX;
     unsigned pushed = 0;
-    for (int base = 0; base < len; base += kBlk) {
-        const int i = base + threadIdx.x;
+    for (int64_t base = lo; base < hi; base += kBlk) {
+        const int64_t i = base + threadIdx.x;
         int32_t v = -1, d = kDead;
-        if (i < len) { v = src[i]; d = deg[v]; }
+        if (i < hi) { v = src[i]; d = deg[v]; }
         const bool fr = d <= k;               // alive (< kDead) and in the k-shell
         const bool keep = d > k && d < kDead;
         if (keep) lmin = min(lmin, d);
+        if (mode) {  // near list: k < deg <= theta
+            const bool nk = keep && d <= theta;
+            const unsigned bn = __ballot_sync(kFull, nk);
+            if (bn) {
+                unsigned long long p2 = 0;
+                if (lane == 0) p2 = atomicAdd(ntail, (unsigned long long)__popc(bn));
+                p2 = __shfl_sync(kFull, p2, 0);
+                if (nk) ndst[p2 + __popc(bn & ((1u << lane) - 1u))] = v;
+            }
+        }
         if (fr) { deg[v] = d + kRemoved; R.core[v] = k; }
         // frontier -> own inbox (local append), survivors -> compacted segment
         const unsigned bf = __ballot_sync(kFull, fr);
@@ -356,7 +396,7 @@ __device__ void phase_scan(const Args &A, Smem &sm, int rl, int b, int k, int se
             if (fr) inbox[p0 + __popc(bf & ((1u << lane) - 1u))] = v;
             pushed += lane == 0 ? __popc(bf) : 0;
         }
-        const unsigned bk = __ballot_sync(kFull, keep);
+        const unsigned bk = __ballot_sync(kFull, keep && dst != nullptr);
         if (bk) {
             int p1 = 0;
             if (lane == 0) p1 = atomicAdd(&sm.kcur, __popc(bk));
@@ -372,7 +412,7 @@ __device__ void phase_scan(const Args &A, Smem &sm, int rl, int b, int k, int se
         int m = INT_MAX;
         for (int w = 0; w < kWarps; w++) m = min(m, sm.red_min[w]);
         if (m != INT_MAX) atom_min(&gctl(sm)->min_next, m, A.sys);
-        R.seglen[sel ^ 1][b] = sm.kcur;
+        if (mode != 2) R.seglen[sel ^ 1][b] = sm.kcur;
     }
     __syncthreads();
 }
@@ -406,6 +446,10 @@ __device__ __forceinline__ unsigned dec_targets4(const Args &A, const Smem &sm, 
             hits++;
         } else if (old[r] > k + 1 && old[r] < kDead) {
             lmin = min(lmin, old[r] - 1);
+            if (old[r] == sm.th1) {  // theta+1 -> theta: the target joins its owner's near list
+                const unsigned long long pos = atom_add64(ntail_of(A, sm, o[r], sm.near_cur), 1ULL, A.sys);
+                near_of(A, sm, o[r], sm.near_cur)[pos] = lu[r];
+            }
         }
     }
     return hits;
@@ -414,7 +458,7 @@ __device__ __forceinline__ unsigned dec_targets4(const Args &A, const Smem &sm, 
 // Walk arcs [a, e) of one owned row with the whole warp; the next batch's
 // colidx loads are in flight while this batch's atomics complete.
 __device__ __forceinline__ void walk_arcs(const Args &A, Smem &sm, const RankLocal &R, int64_t a, int64_t e, int k,
-                                          int par, int &lmin, unsigned long long &walked)
+                                          int par, int &lmin, unsigned long long &walked, unsigned &pushed)
 {
     const int lane = threadIdx.x & 31;
     walked += (unsigned long long)(e - a);
@@ -433,7 +477,7 @@ __device__ __forceinline__ void walk_arcs(const Args &A, Smem &sm, const RankLoc
             const int64_t x = a + 128 + r * 32 + lane;
             un[r] = x < e ? __ldg(R.ci + x) : -1;
         }
-        count_pushed(A, sm, dec_targets4(A, sm, u, k, par, lmin));
+        pushed += dec_targets4(A, sm, u, k, par, lmin);
     }
 }
 
@@ -441,7 +485,8 @@ __device__ __forceinline__ void walk_arcs(const Args &A, Smem &sm, const RankLoc
 // d, exclusive prefix pre over the lanes, total T): 128 arcs per step, each
 // arc finds its row with a 5-step shuffle search -- short rows fill the lanes.
 __device__ __forceinline__ void walk_rows32(const Args &A, Smem &sm, const RankLocal &R, int64_t b, int32_t pre,
-                                            int32_t T, int k, int par, int &lmin, unsigned long long &walked)
+                                            int32_t T, int k, int par, int &lmin, unsigned long long &walked,
+                                            unsigned &pushed)
 {
     const int lane = threadIdx.x & 31;
     walked += (unsigned long long)T;
@@ -460,7 +505,7 @@ __device__ __forceinline__ void walk_rows32(const Args &A, Smem &sm, const RankL
             const int32_t rq = __shfl_sync(kFull, pre, pos);
             u[r] = x < T ? __ldg(R.ci + rb + (x - rq)) : -1;
         }
-        count_pushed(A, sm, dec_targets4(A, sm, u, k, par, lmin));
+        pushed += dec_targets4(A, sm, u, k, par, lmin);
     }
 }
 
@@ -487,6 +532,7 @@ __device__ void phase_peel(const Args &A, Smem &sm, int rl, int k, int par, int 
     unsigned long long *lc = R.lctl;
     int lmin = INT_MAX;
     unsigned long long walked = 0;
+    unsigned pushed = 0;  // counted into the global pushed counter once, at the end
     while (true) {  // items, 32 per pop
         int64_t i0 = 0;
         if (lane == 0) i0 = (int64_t)atomicAdd(&lc[0], 32ULL);
@@ -528,26 +574,11 @@ __device__ void phase_peel(const Args &A, Smem &sm, int rl, int k, int par, int 
                 }
                 const int64_t bj = __shfl_sync(kFull, b, pos), ej = __shfl_sync(kFull, e, pos);
                 const int32_t qj = q - __shfl_sync(kFull, cpre, pos);
-                if (q < ctot) {
-                    const int64_t cb = bj + (int64_t)qj * kChunk;
-                    R.chunk_beg[c0 + q] = cb;
-                }
-            }
-            __threadfence();  // the chunks are read by other CTAs of the rank
-            for (int32_t q0 = 0; q0 < ctot; q0 += 32) {
-                const int32_t q = q0 + lane;
-                int pos = 0;
-#pragma unroll
-                for (int bs = 16; bs >= 1; bs >>= 1) {
-                    const int32_t x = __shfl_sync(kFull, cpre, pos + bs);
-                    if (x <= q) pos += bs;
-                }
-                const int64_t bj = __shfl_sync(kFull, b, pos), ej = __shfl_sync(kFull, e, pos);
-                const int32_t qj = q - __shfl_sync(kFull, cpre, pos);
-                if (q < ctot) {
+                if (q < ctot) {  // descriptor and publication are one atomic word: no fence
                     const int64_t cb = bj + (int64_t)qj * kChunk;
                     const int len = (int)min((int64_t)kChunk, ej - cb);
-                    atomicExch(&R.chunk_tag[c0 + q], ((unsigned)epoch << 12) | (unsigned)(len - 1));
+                    atomicExch(&R.chunk[c0 + q], ((unsigned long long)epoch << 44) |
+                                                     ((unsigned long long)(len - 1) << 36) | (unsigned long long)cb);
                 }
             }
         }
@@ -561,18 +592,18 @@ __device__ void phase_peel(const Args &A, Smem &sm, int rl, int k, int par, int 
             if (lane >= o) incl += t;
         }
         const int32_t T = __shfl_sync(kFull, incl, 31);
-        if (T > 0) walk_rows32(A, sm, R, b, incl - d, T, k, par, lmin, walked);
+        if (T > 0) walk_rows32(A, sm, R, b, incl - d, T, k, par, lmin, walked, pushed);
     }
     peel_mark(A, rec, 4);
     while (true) {  // chunks of long rows
-        int64_t c = 0;
+        unsigned long long w = 0ULL;
         bool done = false;
         if (lane == 0) {
-            c = (int64_t)atomicAdd(&lc[3], 1ULL);
+            const int64_t c = (int64_t)atomicAdd(&lc[3], 1ULL);
             while (true) {
                 const unsigned long long tail = *(volatile unsigned long long *)&lc[2];
                 if ((unsigned long long)c < tail) {
-                    while ((atomicAdd(&R.chunk_tag[c], 0u) >> 12) != (unsigned)epoch) __nanosleep(32);
+                    while (((w = atomicAdd(&R.chunk[c], 0ULL)) >> 44) != (unsigned long long)epoch) __nanosleep(20);
                     break;
                 }
                 if (*(volatile unsigned long long *)&lc[1] >= (unsigned long long)size &&
@@ -580,18 +611,18 @@ __device__ void phase_peel(const Args &A, Smem &sm, int rl, int k, int par, int 
                     done = true;
                     break;
                 }
-                __nanosleep(200);  // back off: idle warps must not slow the working ones down
+                __nanosleep(64);  // back off: idle warps must not slow the working ones down
             }
         }
         done = __shfl_sync(kFull, done, 0);
         if (done) break;
-        c = __shfl_sync(kFull, c, 0);
-        __threadfence();
-        const int64_t cb = R.chunk_beg[c];
-        const int len = (int)(R.chunk_tag[c] & 4095u) + 1;
-        walk_arcs(A, sm, R, cb, cb + len, k, par, lmin, walked);
+        w = __shfl_sync(kFull, w, 0);
+        const int64_t cb = (int64_t)(w & ((1ULL << 36) - 1ULL));
+        const int len = (int)((w >> 36) & 255ULL) + 1;
+        walk_arcs(A, sm, R, cb, cb + len, k, par, lmin, walked, pushed);
     }
     peel_mark(A, rec, 5);
+    count_pushed(A, sm, pushed);  // before the barrier reads the counter
     if (A.trace && (threadIdx.x & 31) == 0 && rec < A.trace_cap && walked) {  // latest end of any walking warp
         unsigned long long t;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -631,18 +662,39 @@ __global__ void __launch_bounds__(kBlk, 1) k_mgd(const __grid_constant__ Args A)
     tr(1, 0, 0);
     int k = -1, sel = 0, par = 0, epoch = 1;
     int64_t levels = sm.snap_pushed > 0 ? 1 : 0;  // the 0-shell (isolated vertices, removed at INIT)
-    int64_t subrounds = 0, barriers = 1, kmax = 0;
+    int64_t subrounds = 0, barriers = 1, kmax = 0, near_scans = 0;
+    bool near_on = false;
+    int theta = 0;
+    if (threadIdx.x == 0) { sm.th1 = INT_MIN; sm.near_cur = 0; }
+    __syncthreads();
     while (true) {
         if (sm.snap_pushed >= (unsigned long long)A.n) break;  // every vertex removed
-        k = max(k + 1, sm.snap_min);
+        // level skip (R5); inside a near epoch every vertex outside the list has deg > theta
+        k = near_on ? max(k + 1, min(sm.snap_min, theta + 1)) : max(k + 1, sm.snap_min);
         const unsigned long long before = sm.snap_pushed;
-        phase_scan(A, sm, rl, b, k, sel, par);
-        sel ^= 1;
-        gbar(A, sm, rl, -1, 1);
+        int mode, near_reset = -1;
+        if (near_on && k <= theta) {
+            mode = 2;  // near scan: consumes near[cur]
+            near_reset = sm.near_cur;
+            near_scans++;
+        } else {
+            near_on = (int64_t)(A.n - (int64_t)sm.snap_pushed) >= kNearMin;  // uniform decision
+            theta = near_on ? (int)min((int64_t)INT_MAX - 2, (int64_t)k + kNearW) : 0;
+            mode = near_on ? 1 : 0;
+            if (near_on) near_reset = sm.near_cur;  // the previous epoch's list is dropped
+        }
+        phase_scan(A, sm, rl, b, k, sel, par, mode, theta);
+        if (mode != 2) sel ^= 1;
+        gbar(A, sm, rl, -1, 1, near_reset);
+        if (threadIdx.x == 0) {
+            if (mode) sm.near_cur ^= 1;  // the list this scan wrote is current; walks append to it
+            sm.th1 = near_on ? theta + 1 : INT_MIN;
+        }
+        __syncthreads();
         barriers++;
         tr(barriers, 1, k);
         while (sm.snap_pushed != sm.snap_prev) {  // something was pushed: walk it
-            phase_peel(A, sm, rl, k, par, epoch++ & 0xfffff, barriers + 1);
+            phase_peel(A, sm, rl, k, par, 1 + (epoch++ % 0xfffff), barriers + 1);  // 20-bit epochs, never 0
             peel_mark(A, barriers + 1, 6);
             gbar(A, sm, rl, par, 1);  // the consumed inbox tail is reset by the rank's last arriver
             par ^= 1;
@@ -658,6 +710,7 @@ __global__ void __launch_bounds__(kBlk, 1) k_mgd(const __grid_constant__ Args A)
         A.stats[2] = barriers;
         A.stats[3] = kmax;
         A.stats[4] = (int64_t)*(volatile unsigned long long *)&gctl(sm)->arcs;
+        A.stats[5] = near_scans;
     }
 }
 
@@ -695,7 +748,7 @@ namespace {
 size_t al256(size_t x) { return (x + 255) & ~(size_t)255; }
 
 struct Layout {
-    int64_t off_tail, off_deg, off_in0, off_in1, in_cap;
+    int64_t off_tail, off_deg, off_in0, off_in1, off_near0, off_near1, in_cap;
     size_t bytes;
 };
 
@@ -711,6 +764,10 @@ Layout window_layout(int64_t nl_max)
     L.off_in0 = (int64_t)off;
     off += al256(sizeof(int32_t) * (size_t)nn);
     L.off_in1 = (int64_t)off;
+    off += al256(sizeof(int32_t) * (size_t)nn);
+    L.off_near0 = (int64_t)off;
+    off += al256(sizeof(int32_t) * (size_t)nn);
+    L.off_near1 = (int64_t)off;
     off += al256(sizeof(int32_t) * (size_t)nn);
     L.in_cap = nn;
     L.bytes = off;
@@ -733,20 +790,18 @@ int setup_local(mgd::RankLocal &R, int G, int64_t m_local, cudaStream_t st, void
     const size_t o_alive1 = off; off += al256(sizeof(int32_t) * (size_t)(seg_cap * G));
     const size_t o_seg0 = off; off += al256(sizeof(int32_t) * (size_t)G);
     const size_t o_seg1 = off; off += al256(sizeof(int32_t) * (size_t)G);
-    const size_t o_cb = off; off += al256(sizeof(int64_t) * (size_t)chunk_cap);
-    const size_t o_ct = off; off += al256(sizeof(int32_t) * (size_t)chunk_cap);
+    const size_t o_cb = off; off += al256(sizeof(unsigned long long) * (size_t)chunk_cap);
     const size_t o_lc = off; off += 256;
     char *m = nullptr;
     MGD_CK(cudaMallocAsync((void **)&m, off, st));
-    MGD_CK(cudaMemsetAsync(m + o_ct, 0, sizeof(int32_t) * (size_t)chunk_cap, st));
+    MGD_CK(cudaMemsetAsync(m + o_cb, 0, sizeof(unsigned long long) * (size_t)chunk_cap, st));
     MGD_CK(cudaMemsetAsync(m + o_lc, 0, 256, st));  // rank-local cursors and barrier words
     R.alive[0] = (int32_t *)(m + o_alive0);
     R.alive[1] = (int32_t *)(m + o_alive1);
     R.seglen[0] = (int32_t *)(m + o_seg0);
     R.seglen[1] = (int32_t *)(m + o_seg1);
     R.seg_cap = seg_cap;
-    R.chunk_beg = (int64_t *)(m + o_cb);
-    R.chunk_tag = (uint32_t *)(m + o_ct);
+    R.chunk = (unsigned long long *)(m + o_cb);
     R.chunk_cap = chunk_cap;
     R.lctl = (unsigned long long *)(m + o_lc);
     *mem_out = m;
@@ -781,6 +836,7 @@ int launch(mgd::Args &A, cudaStream_t st, kcore_stats *stats, int64_t *d_stats, 
         stats->barriers = hs[2];
         stats->kmax = (int32_t)hs[3];
         stats->arcs_walked = hs[4];
+        stats->near_scans = hs[5];
         stats->grid_blocks = A.PL * A.G;
         stats->block_threads = mgd::kBlk;
         stats->kernel_ms = ms;
@@ -843,6 +899,7 @@ int mgd_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t
         for (int r = 0; r < nranks; r++) nl_max = std::max<int64_t>(nl_max, A->vb[r + 1] - A->vb[r]);
         const Layout L = window_layout(nl_max);
         A->off_tail = L.off_tail; A->off_deg = L.off_deg; A->off_in0 = L.off_in0; A->off_in1 = L.off_in1;
+        A->off_near0 = L.off_near0; A->off_near1 = L.off_near1;
         A->in_cap = L.in_cap;
         MGD_CK(cudaMallocAsync((void **)&slab, L.bytes * nranks, st));
         MGD_CK(cudaMemsetAsync(slab, 0, L.bytes * nranks, st));
@@ -934,6 +991,7 @@ int mgd_nccl(const int64_t *rowptr_local, const int32_t *colidx_local, int64_t n
         for (int r = 0; r < P; r++) nl_max = std::max<int64_t>(nl_max, A->vb[r + 1] - A->vb[r]);
         const Layout L = window_layout(nl_max);
         A->off_tail = L.off_tail; A->off_deg = L.off_deg; A->off_in0 = L.off_in0; A->off_in1 = L.off_in1;
+        A->off_near0 = L.off_near0; A->off_near1 = L.off_near1;
         A->in_cap = L.in_cap;
         if (ncclMemAlloc(&win_mem, L.bytes) != ncclSuccess) { rc = KCORE_ENCCL; goto out; }
         MGD_CK(cudaMemsetAsync(win_mem, 0, L.bytes, st));

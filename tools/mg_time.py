@@ -31,13 +31,18 @@ for name in a.cfgs:
         ms, st = [], None
         for rep in range(6):
             flush.fill_(1)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
             got, st = kc.kcore_decompose_mg_virtual(r, c, P, stats=True, algo=a.algo)
+            e1.record()
+            torch.cuda.synchronize()
             if rep == 0:
                 assert torch.equal(got, ref), (name, P)
                 continue
-            ms.append(st.kernel_ms if a.algo == 0 else 0.0)
+            # device protocol: the kernel's own events; host-driven: the whole call (it syncs per sub-round)
+            ms.append(st.kernel_ms if a.algo == 0 else e0.elapsed_time(e1))
         res[f"P{P}"] = {"ms": statistics.median(ms), "subrounds": st.phases, "barriers": st.barriers,
-                        "levels": st.levels}
+                        "levels": st.levels, "near_scans": st.near_scans}
         print(name, P, res[f"P{P}"], "single", res["single_ms"], flush=True)
     out[name] = res
     del r, c, ref
