@@ -145,11 +145,19 @@ def run_reference(args):
 
 
 def _lib_sha():
+    """Identity of the benchmarked kernel's code: sha256 of the SASS
+    instruction lines of k_persistent (cuobjdump).  Unlike the .so's own hash it is the same for every build
+    of the same sources (nvcc embeds build-specific bytes in the fat binary)."""
     import hashlib
+    import re
     try:
         import paper_conf_icde_ahmady0gcz23_b200 as kc
-        with open(kc.LIB_PATH, "rb") as f:
-            return hashlib.sha256(f.read()).hexdigest()
+        out = subprocess.run(["cuobjdump", "-sass", "-fun", "_ZN2kc12k_persistentENS_5KArgsE", kc.LIB_PATH],
+                             capture_output=True, text=True, timeout=120).stdout
+        lines = [ln for ln in out.splitlines() if re.match(r"^\s+/\*[0-9a-f]{4,}\*/", ln)]
+        if not lines:
+            return None
+        return hashlib.sha256("\n".join(lines).encode()).hexdigest()
     except Exception:
         return None
 
@@ -317,8 +325,8 @@ def run_gpu(args):
     b_min = 4 * m_arcs + 8 * (n + 1) + 8 * n + 4 * n + 4 * scanned + 8 * n  # SURVEY 8(d) B_min
     achieved = b_min / (kern_ms * 1e-3) / 1e9
     # DRAM traffic of the dominant kernel: from the committed `ncu --set full`
-    # capture ONLY if that capture profiled this very library binary (sha256
-    # recorded in the capture); otherwise null.  (ncu cannot run inside the
+    # capture ONLY if that capture profiled this very device code (sha256 of
+    # the SASS, recorded in the capture); otherwise null.  (ncu cannot run inside the
     # timed bench; profiles/README.md has the capture command.)
     traffic, traffic_src = None, None
     lib_sha = _lib_sha()
@@ -326,9 +334,9 @@ def run_gpu(args):
     if os.path.exists(tpath) and world == 1 and not args.force_mg:
         try:
             tj = json.load(open(tpath))
-            if tj.get("lib_sha256") == lib_sha:
+            if lib_sha and tj.get("sass_sha256") == lib_sha:
                 traffic = tj.get("dram_bytes_per_launch")
-                traffic_src = {"file": "profiles/ncu_traffic_C4.json", "lib_sha256": lib_sha,
+                traffic_src = {"file": "profiles/ncu_traffic_C4.json", "sass_sha256": lib_sha,
                                "window_off_bytes": tj.get("dram_bytes_per_launch_window_off")}
         except Exception:
             traffic = None
@@ -348,7 +356,7 @@ def run_gpu(args):
                    "step_ms_std": statistics.pstdev(step_ms) if len(step_ms) > 1 else 0.0,
                    "kernel_ms_median": statistics.median(s.kernel_ms for s in stats),
                    "kernel_ms_min": min(s.kernel_ms for s in stats)},
-        "lib_sha256": lib_sha,
+        "sass_sha256": lib_sha,
         "gpu_launches": int(sum(s.launches for s in stats)),  # counted by the library, timed steps only
         "e2e": e2e,
         "clocks": clk,

@@ -1,7 +1,7 @@
 """Write profiles/ncu_traffic_C4.json (bench.py's roofline.traffic source) from
 an ncu --set full capture and a window-off metrics CSV of the SAME library
 binary: python tools/traffic_json.py DIR  (DIR holds prof_C4.ncu-rep,
-ncu_window_off.csv, lib_sha.txt as written by tools/gpu/final.sh)."""
+ncu_window_off.csv, sass_sha.txt as written by tools/gpu/final.sh)."""
 import csv
 import io
 import json
@@ -29,9 +29,9 @@ for line in open(os.path.join(d, "ncu_window_off.csv")):
         continue
     f = next(csv.reader([line]))
     off[f[-3]] = float(f[-1])
-sha = open(os.path.join(d, "lib_sha.txt")).read().split()[0]
+sha = open(os.path.join(d, "sass_sha.txt")).read().split()[0]
 out = {
-    "lib_sha256": sha,
+    "sass_sha256": sha,
     "kernel": "k_persistent(KArgs)", "config": "C4 rmat-s24-ef32",
     "dram_bytes_per_launch": val("dram__bytes_read.sum") + val("dram__bytes_write.sum"),
     "dram_bytes_read": val("dram__bytes_read.sum"), "dram_bytes_write": val("dram__bytes_write.sum"),
