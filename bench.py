@@ -280,10 +280,13 @@ def run_gpu(args):
         dist.barrier()
     step_ms = [a.elapsed_time(b) for a, b in evs]
     total_ms = sum(step_ms)
+    per_rank_ms = None
     if world > 1:
         t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
+        allt = [torch.zeros_like(t) for _ in range(world)]
+        dist.all_gather(allt, t)
+        per_rank_ms = [float(x.item()) / args.steps for x in allt]  # per step, every rank
+        total_ms = max(float(x.item()) for x in allt)  # the job's time: the slowest rank
     value = args.steps * m_und / (total_ms * 1e-3) / 1e6
     ms_per_step = total_ms / args.steps
 
@@ -362,6 +365,7 @@ def run_gpu(args):
         "clocks": clk,
         "stats": {"levels": st.levels, "phases": st.phases, "barriers": st.barriers, "scanned": st.scanned,
                   "kmax": st.kmax, "grid": st.grid_blocks, "block": st.block_threads},
+        "per_rank_ms_per_step": per_rank_ms,
     }
     if world == 1 and not args.force_mg and not args.no_mpm:
         # the paper's second algorithm family on the same graph: MPM h-index
