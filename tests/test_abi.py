@@ -104,3 +104,18 @@ def test_no_cpu_fallback_in_product_package():
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "networkx" not in src, f
+
+
+def test_committed_traffic_capture_matches_kernel_code():
+    """profiles/ncu_traffic_C4.json (bench.py's roofline.traffic) was captured on
+    exactly the k_persistent code this tree builds (sha256 of its SASS)."""
+    import json
+    import shutil
+    import bench
+    if shutil.which("cuobjdump") is None:
+        pytest.skip("cuobjdump not available")
+    sha = bench._lib_sha()
+    assert sha and len(sha) == 64
+    tj = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic_C4.json")))
+    assert tj["sass_sha256"] == sha
+    assert tj["dram_bytes_per_launch"] > 0 and tj["dram_bytes_per_launch_window_off"] > 0
