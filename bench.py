@@ -11,9 +11,11 @@ device-resident CSR.  Between steps L2 is flushed (a 512 MiB write) outside
 the timed events.  value = undirected edges / step time (Medges/s), summed
 over K steps, max over ranks for N > 1.
 
-N > 1 runs the multi-GPU protocol (kcore_decompose_mg, 1-D vertex ranges,
-NCCL between ranks) on the same graph: strong scaling (the workload is one
-fixed graph at every N, so every line says "strong").
+N > 1 runs the multi-GPU protocol on the same graph (1-D vertex ranges): by
+default the device-initiated kernel over NCCL symmetric memory
+(kcore_decompose_mg_ex(KCORE_MG_DEVICE)), --mg-algo host the host-driven NCCL
+exchange.  Strong scaling (the workload is one fixed graph at every N, so
+every line says "strong").
 
 --impl reference times the CPU oracle (serial Batagelj-Zaversnik, oracle/)
 on the host, each step a bounded sample of the workload (R-MAT scale 22,
@@ -350,7 +352,8 @@ def run_gpu(args):
         "data": "synthetic",
         "config": {"workload": WORKLOAD, "baseline_config": "BASELINE.json configs[3]", "n": n,
                    "m_undirected": m_und, "arcs": m_arcs, "l2": "flushed between steps (512 MiB write); "
-                   "colidx 4 GB > L2", "parallelism": f"vertex-range x{world}" if world > 1 else "1 GPU"},
+                   "colidx 4 GB > L2", "parallelism": (f"vertex-range x{world} ({args.mg_algo})" if world > 1 or args.force_mg
+                                                    else "1 GPU")},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "traffic_source": traffic_src,
                      "peak_source": peak_src, "algorithmic_bytes": b_min, "kernel_ms": kern_ms},
@@ -434,8 +437,9 @@ def main():
     ap.add_argument("--no-mpm", action="store_true", help="skip the MPM context measurement")
     ap.add_argument("--force-mg", action="store_true", help="run the multi-GPU path even at N=1")
     ap.add_argument("--no-configs", action="store_true", help="skip the C1-C3 per-config measurements")
-    ap.add_argument("--mg-algo", default="host", choices=["host", "device"],
-                    help="N > 1: host-driven NCCL exchange (default) or the device-initiated kernel")
+    ap.add_argument("--mg-algo", default="device", choices=["host", "device"],
+                    help="N > 1: the device-initiated kernel over NCCL symmetric memory (default, SURVEY f1) "
+                         "or the host-driven NCCL exchange per sub-round")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
