@@ -25,6 +25,11 @@ extern "C" {
 int kcore_test_ballot_compact(const int32_t *vid, const int32_t *pred, int32_t n, int32_t *prefix,
                               int32_t *buf, int32_t *e, void *stream);
 
+/* Watchdog of the device-initiated multi-GPU kernel: every wait longer than
+ * `ns` nanoseconds aborts the call with KCORE_ECUDA instead of hanging
+ * (default 60 s; ns <= 0 restores it).  Tests shorten it to exercise the path. */
+int kcore_test_mgd_timeout(int64_t ns);
+
 /* Phase trace of the next kcore_decompose_mg_virtual call (device-initiated
  * protocol; development aid): DEVICE int64[cap][4] records {globaltimer ns,
  * phase (-1 start, 0 init, 1 scan, 2 sub-round), k, removed so far} at every

@@ -80,6 +80,7 @@ struct Ctl {  // rank 0's copy is the global control block
     unsigned long long snap_pushed;
     unsigned long long snap_prev;  // pushed at the previous barrier
     int snap_par;
+    alignas(128) int abort;        // watchdog: a CTA waited past the deadline (every CTA leaves)
 };
 
 struct RankLocal {
@@ -110,6 +111,7 @@ struct Args {
     int64_t off_tail, off_deg, off_in0, off_in1, in_cap;
     int64_t off_near0, off_near1;  // near lists [2][nl_max] (their tails follow the inbox tails)
     int64_t *stats;     // [0] levels [1] sub-rounds [2] barriers [3] kmax [4] arcs
+    int64_t timeout_ns; // watchdog: a wait longer than this aborts the call (KCORE_ECUDA), 0 = none
     int64_t *trace;     // optional [trace_cap][8]: {globaltimer, phase (0 init 1 scan 2 peel), k, pushed,
                         //  block 0's peel: items done, chunks done, end}
     int64_t trace_cap;
@@ -124,6 +126,8 @@ struct Smem {
     unsigned long long snap_pushed, snap_prev;
     int snap_min, snap_par;
     float inv_n;  // P / n
+    unsigned long long deadline;  // globaltimer deadline of the watchdog
+    int aborted;
     int th1;      // theta + 1 of the running near epoch (INT_MIN: none): walks append theta+1 -> theta crossings
     int near_cur; // near[near_cur] is the list the next near scan reads (and walks append to)
 };
@@ -191,7 +195,24 @@ __device__ __forceinline__ unsigned long long *ntail_of(const Args &A, const Sme
 // always take the level minimum; mode 1: take it (and end the level) only if
 // nothing was pushed since the previous barrier.
 enum : int { L_POP = 0, L_DONE = 1, L_CTAIL = 2, L_CPOP = 3, L_BAR = 4, L_GEN = 5, L_SPUSH = 6, L_SPREV = 7,
-             L_SMIN = 8 };
+             L_SMIN = 8, L_ABORT = 9 };
+
+// Watchdog of every wait (the multi-GPU protocol has not run on several GPUs
+// yet): past the deadline, or once any CTA gave up, the waiter leaves, the
+// kernel returns and the host reports KCORE_ECUDA instead of hanging.
+__device__ __noinline__ bool watchdog(const Args &A, Smem &sm)
+{
+    if (A.timeout_ns <= 0) return false;
+    Ctl *c = (Ctl *)sm.peer[0];
+    if (*(volatile int *)&c->abort) return true;
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t > sm.deadline) {
+        *(volatile int *)&c->abort = 1;
+        return true;
+    }
+    return false;
+}
 
 // Virtual ranks (one launch holds every rank): a single-level barrier over all
 // P*G CTAs; the last arriver resets every rank's cursors itself.
@@ -222,7 +243,8 @@ __device__ void gbar_flat(const Args &A, Smem &sm, int reset_par, int mode, int 
             __threadfence();
             *(volatile unsigned *)&c->bar_gen = gen + 1u;
         } else {
-            while (ld_volatile_u32(&c->bar_gen) == gen) {
+            for (unsigned it = 1; ld_volatile_u32(&c->bar_gen) == gen; it++) {
+                if ((it & 1023u) == 0u && watchdog(A, sm)) { sm.aborted = 1; break; }
             }
             __threadfence();
         }
@@ -269,7 +291,8 @@ __device__ void gbar(const Args &A, Smem &sm, int rl, int reset_par, int mode, i
                 fence(sys);
                 *(volatile unsigned *)&c->bar_gen = gen + 1u;
             } else {
-                while (ld_volatile_u32(&c->bar_gen) == gen) {
+                for (unsigned it = 1; ld_volatile_u32(&c->bar_gen) == gen; it++) {
+                    if ((it & 1023u) == 0u && watchdog(A, sm)) { sm.aborted = 1; break; }
                 }
                 fence(sys);
             }
@@ -279,7 +302,8 @@ __device__ void gbar(const Args &A, Smem &sm, int rl, int reset_par, int mode, i
             __threadfence();
             *(volatile unsigned long long *)&lc[L_GEN] = lgen + 1ULL;
         } else {
-            while (*(volatile unsigned long long *)&lc[L_GEN] == lgen) {
+            for (unsigned it = 1; *(volatile unsigned long long *)&lc[L_GEN] == lgen; it++) {
+                if ((it & 1023u) == 0u && watchdog(A, sm)) { sm.aborted = 1; break; }
             }
             __threadfence();
         }
@@ -600,10 +624,16 @@ __device__ void phase_peel(const Args &A, Smem &sm, int rl, int k, int par, int 
         bool done = false;
         if (lane == 0) {
             const int64_t c = (int64_t)atomicAdd(&lc[3], 1ULL);
+            unsigned spins = 0;
             while (true) {
                 const unsigned long long tail = *(volatile unsigned long long *)&lc[2];
                 if ((unsigned long long)c < tail) {
-                    while (((w = atomicAdd(&R.chunk[c], 0ULL)) >> 44) != (unsigned long long)epoch) __nanosleep(20);
+                    bool gone = false;
+                    for (unsigned it = 1; ((w = atomicAdd(&R.chunk[c], 0ULL)) >> 44) != (unsigned long long)epoch; it++) {
+                        __nanosleep(20);
+                        if ((it & 1023u) == 0u && watchdog(A, sm)) { gone = true; break; }
+                    }
+                    if (gone) { sm.aborted = 1; done = true; }
                     break;
                 }
                 if (*(volatile unsigned long long *)&lc[1] >= (unsigned long long)size &&
@@ -612,6 +642,7 @@ __device__ void phase_peel(const Args &A, Smem &sm, int rl, int k, int par, int 
                     break;
                 }
                 __nanosleep(64);  // back off: idle warps must not slow the working ones down
+                if ((++spins & 255u) == 0u && watchdog(A, sm)) { sm.aborted = 1; done = true; break; }
             }
         }
         done = __shfl_sync(kFull, done, 0);
@@ -646,7 +677,13 @@ __global__ void __launch_bounds__(kBlk, 1) k_mgd(const __grid_constant__ Args A)
     const int rl = blockIdx.x / A.G, b = blockIdx.x % A.G;
     if (threadIdx.x < kMaxR) sm.peer[threadIdx.x] = A.peer_dev ? A.peer_dev[threadIdx.x] : A.peer[threadIdx.x];
     if (threadIdx.x <= kMaxR) sm.vb[threadIdx.x] = A.vb[threadIdx.x];
-    if (threadIdx.x == 0) sm.inv_n = (float)A.P / (float)(A.n > 0 ? A.n : 1);
+    if (threadIdx.x == 0) {
+        sm.inv_n = (float)A.P / (float)(A.n > 0 ? A.n : 1);
+        unsigned long long t;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        sm.deadline = t + (unsigned long long)A.timeout_ns;
+        sm.aborted = 0;
+    }
     __syncthreads();
     auto tr = [&](int64_t i, int ph, int k) {
         if (A.trace && blockIdx.x == 0 && threadIdx.x == 0 && i < A.trace_cap) {
@@ -659,6 +696,7 @@ __global__ void __launch_bounds__(kBlk, 1) k_mgd(const __grid_constant__ Args A)
     tr(0, -1, 0);
     phase_init(A, sm, rl, b);
     gbar(A, sm, rl, -1, 0);
+    if (sm.aborted) { if (threadIdx.x == 0) A.R[rl].lctl[L_ABORT] = 1ULL; return; }
     tr(1, 0, 0);
     int k = -1, sel = 0, par = 0, epoch = 1;
     int64_t levels = sm.snap_pushed > 0 ? 1 : 0;  // the 0-shell (isolated vertices, removed at INIT)
@@ -686,6 +724,7 @@ __global__ void __launch_bounds__(kBlk, 1) k_mgd(const __grid_constant__ Args A)
         phase_scan(A, sm, rl, b, k, sel, par, mode, theta);
         if (mode != 2) sel ^= 1;
         gbar(A, sm, rl, -1, 1, near_reset);
+        if (sm.aborted) { if (threadIdx.x == 0) A.R[rl].lctl[L_ABORT] = 1ULL; return; }
         if (threadIdx.x == 0) {
             if (mode) sm.near_cur ^= 1;  // the list this scan wrote is current; walks append to it
             sm.th1 = near_on ? theta + 1 : INT_MIN;
@@ -697,6 +736,7 @@ __global__ void __launch_bounds__(kBlk, 1) k_mgd(const __grid_constant__ Args A)
             phase_peel(A, sm, rl, k, par, 1 + (epoch++ % 0xfffff), barriers + 1);  // 20-bit epochs, never 0
             peel_mark(A, barriers + 1, 6);
             gbar(A, sm, rl, par, 1);  // the consumed inbox tail is reset by the rank's last arriver
+            if (sm.aborted) { if (threadIdx.x == 0) A.R[rl].lctl[L_ABORT] = 1ULL; return; }
             par ^= 1;
             subrounds++;
             barriers++;
@@ -809,9 +849,12 @@ out:
     return rc;
 }
 
-int launch(mgd::Args &A, cudaStream_t st, kcore_stats *stats, int64_t *d_stats, int64_t launches)
+int launch(mgd::Args &A, cudaStream_t st, kcore_stats *stats, int64_t *d_stats, int64_t launches,
+           int64_t timeout_ns)
 {
     int rc = KCORE_OK;
+    // watchdog: no wait of the protocol may exceed a minute (tests may shorten it)
+    A.timeout_ns = timeout_ns > 0 ? timeout_ns : (int64_t)60 * 1000000000LL;
     cudaEvent_t e0 = nullptr, e1 = nullptr;
     int64_t hs[8] = {0};
     A.stats = d_stats;
@@ -842,6 +885,15 @@ int launch(mgd::Args &A, cudaStream_t st, kcore_stats *stats, int64_t *d_stats, 
         stats->kernel_ms = ms;
         stats->launches = launches;
     }
+    {  // a CTA that hit the watchdog marked its rank: report an error, do not hang
+        unsigned long long ab = 0;
+        for (int r = 0; r < A.PL && !rc; r++) {
+            MGD_CK(cudaMemcpyAsync(&ab, A.R[r].lctl + mgd::L_ABORT, sizeof(ab), cudaMemcpyDeviceToHost, st));
+            MGD_CK(cudaStreamSynchronize(st));
+            if (ab) rc = KCORE_ECUDA;
+        }
+        if (rc) goto out;
+    }
 out:
     if (e0) cudaEventDestroy(e0);
     if (e1) cudaEventDestroy(e1);
@@ -850,8 +902,15 @@ out:
 
 } // namespace
 
+static int64_t g_timeout_ns = 0;    // kcore_test_mgd_timeout: watchdog override (tests), 0 = default
 static int64_t *g_trace = nullptr;  // kcore_test_mgd_trace: phase trace of the next call (dev aid)
 static int64_t g_trace_cap = 0;
+
+extern "C" int kcore_test_mgd_timeout(int64_t ns)
+{
+    g_timeout_ns = ns > 0 ? ns : 0;
+    return KCORE_OK;
+}
 
 extern "C" int kcore_test_mgd_trace(int64_t *trace, int64_t cap)
 {
@@ -920,7 +979,7 @@ int mgd_virtual(const int64_t *rowptr, const int32_t *colidx, int64_t n, int64_t
     MGD_CK(cudaMallocAsync((void **)&d_stats, sizeof(int64_t) * 8, st));
     A->trace = g_trace;
     A->trace_cap = g_trace_cap;
-    rc = launch(*A, st, stats, d_stats, 2);
+    rc = launch(*A, st, stats, d_stats, 2, g_timeout_ns);
 out:
     for (void *p : locals) if (p) cudaFreeAsync(p, st);
     if (slab) cudaFreeAsync(slab, st);
@@ -1026,7 +1085,7 @@ int mgd_nccl(const int64_t *rowptr_local, const int32_t *colidx_local, int64_t n
         if (rc) goto out;
     }
     MGD_CK(cudaMallocAsync((void **)&d_stats, sizeof(int64_t) * 8, st));
-    rc = launch(*A, st, stats, d_stats, 3);
+    rc = launch(*A, st, stats, d_stats, 3, g_timeout_ns);
 out:
     if (cudaStreamSynchronize(st) != cudaSuccess && !rc) rc = KCORE_ECUDA;
     if (win) ncclCommWindowDeregister(comm, win);
