@@ -1626,7 +1626,15 @@ __device__ __forceinline__ void setup_near(Ctrl &c, const Snap &sn, const Params
 
 // The pure transition function (Alg. 1 l.5-9 and the level skip).  Every CTA
 // applies it to identical inputs, so all copies stay identical.
-__device__ __noinline__ void advance(Ctrl &c, const Snap &sn, const Params &p)
+#ifndef KC_ADV_REG
+#define KC_ADV_REG 1  // advance() on a register copy of the control state (not field by field in shared memory)
+#endif
+#if KC_ADV_REG
+__device__ __forceinline__
+#else
+__device__ __noinline__
+#endif
+void advance(Ctrl &c, const Snap &sn, const Params &p)
 {
     const int64_t gcnt = (int64_t)(sn.gq >> kArcBits), garc = (int64_t)(sn.gq & kArcMask);
     const int64_t removed = (int64_t)sn.ord;
@@ -1868,7 +1876,14 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant_
                 PROBE(36, 0);
                 if (blockIdx.x == 0) trace_rec(S, sm.ctrl, sm.snap, 1);
                 sm.ctrl.st_bar++;
+#if KC_ADV_REG
+                Ctrl cc = sm.ctrl;
+                const Snap sn = sm.snap;
+                advance(cc, sn, p);
+                sm.ctrl = cc;
+#else
                 advance(sm.ctrl, sm.snap, p);
+#endif
                 PROBE(37, 0);
             }
         }
