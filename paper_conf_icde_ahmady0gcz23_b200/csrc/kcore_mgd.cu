@@ -214,12 +214,25 @@ __device__ __noinline__ bool watchdog(const Args &A, Smem &sm)
     return false;
 }
 
+// deadline check at a barrier's entry (no memory traffic: the local deadline only)
+__device__ __forceinline__ bool past_deadline(const Args &A, const Smem &sm)
+{
+    if (A.timeout_ns <= 0) return false;
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t > sm.deadline;
+}
+
 // Virtual ranks (one launch holds every rank): a single-level barrier over all
 // P*G CTAs; the last arriver resets every rank's cursors itself.
 __device__ void gbar_flat(const Args &A, Smem &sm, int reset_par, int mode, int near_reset)
 {
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (threadIdx.x == 0 && past_deadline(A, sm)) {  // leave without arriving: every waiter times out too
+        *(volatile int *)&gctl(sm)->abort = 1;
+        sm.aborted = 1;
+    }
+    if (threadIdx.x == 0 && !sm.aborted) {
         Ctl *c = gctl(sm);
         const unsigned gen = ld_volatile_u32(&c->bar_gen);
         __threadfence();
@@ -262,7 +275,11 @@ __device__ void gbar(const Args &A, Smem &sm, int rl, int reset_par, int mode, i
         return;
     }
     __syncthreads();
-    if (threadIdx.x == 0) {
+    if (threadIdx.x == 0 && past_deadline(A, sm)) {
+        *(volatile int *)&gctl(sm)->abort = 1;
+        sm.aborted = 1;
+    }
+    if (threadIdx.x == 0 && !sm.aborted) {
         const bool sys = A.sys;
         unsigned long long *lc = A.R[rl].lctl;
         const unsigned long long lgen = *(volatile unsigned long long *)&lc[L_GEN];

@@ -109,16 +109,16 @@ def test_nccl_transport_single_rank():
 
 
 def test_device_protocol_watchdog_aborts_instead_of_hanging():
-    """With a 1 us watchdog every barrier wait times out: the call must return
-    KCORE_ECUDA (no hang), and the next call with the default watchdog must
-    succeed and be exact."""
+    """With a 1 ns watchdog the first device barrier is past its deadline: the
+    call must return KCORE_ECUDA (no hang), and the next call with the default
+    watchdog must succeed and be exact."""
     import ctypes
     lib = kc.library()
     lib.kcore_test_mgd_timeout.argtypes = [ctypes.c_int64]
     rp, ci = kcgen.generate_host(kcgen.rmat(12, 16, seed=3))
     ref = oracle.bz_core(rp, ci)
     r, c = _dev(rp, ci)
-    lib.kcore_test_mgd_timeout(1000)
+    lib.kcore_test_mgd_timeout(1)
     try:
         with pytest.raises(kc.KcoreError):
             kc.kcore_decompose_mg_virtual(r, c, 4)
