@@ -12,7 +12,7 @@ PKG     := paper_conf_icde_ahmady0gcz23_b200
 
 KCORE_SRC := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cuh) $(wildcard include/*.h)
 
-all: oracle/liboracle.so kcgen/libkcgen.so $(PKG)/lib/libkcore.so
+all: oracle/liboracle.so kcgen/libkcgen.so $(PKG)/lib/libkcore.so $(PKG)/lib/libkcore_trace.so
 
 oracle/liboracle.so: oracle/kcore_oracle.c
 	gcc -O2 -std=c11 -shared -fPIC $< -o $@
@@ -29,7 +29,14 @@ $(PKG)/lib/libkcore.so: $(KCORE_SRC)
 	    $(PKG)/csrc/kcore.cu $(PKG)/csrc/kcore_mg.cu $(PKG)/csrc/kcore_extract.cu $(PKG)/csrc/kcore_mpm.cu $(PKG)/csrc/kcore_testhooks.cu $(PKG)/csrc/kcore_mgd.cu -o $@ \
 	    -L$(NCCL_DIR)/lib -l:libnccl.so.2 -Xlinker -rpath=$(NCCL_DIR)/lib 2> $(PKG)/lib/ptxas.log || (cat $(PKG)/lib/ptxas.log; false)
 
+# the same library with the per-phase / per-CTA trace compiled in (tools/cta_trace.py)
+$(PKG)/lib/libkcore_trace.so: $(KCORE_SRC)
+	mkdir -p $(PKG)/lib
+	$(NVCC) $(NVFLAGS) -DKC_TRACE=1 -Iinclude -I$(NCCL_DIR)/include -shared \
+	    $(PKG)/csrc/kcore.cu $(PKG)/csrc/kcore_mg.cu $(PKG)/csrc/kcore_extract.cu $(PKG)/csrc/kcore_mpm.cu $(PKG)/csrc/kcore_testhooks.cu $(PKG)/csrc/kcore_mgd.cu -o $@ \
+	    -L$(NCCL_DIR)/lib -l:libnccl.so.2 -Xlinker -rpath=$(NCCL_DIR)/lib
+
 clean:
-	rm -f oracle/liboracle.so kcgen/libkcgen.so $(PKG)/lib/libkcore.so
+	rm -f oracle/liboracle.so kcgen/libkcgen.so $(PKG)/lib/libkcore.so $(PKG)/lib/libkcore_trace.so
 
 .PHONY: all clean

@@ -100,7 +100,9 @@ typedef struct {
                              /* frontiers; a degeneracy order)          */
     void *workspace;         /* optional DEVICE scratch of >= kcore_workspace_size()    */
     size_t workspace_bytes;
-    int64_t *trace_out;      /* optional DEVICE int64[trace_cap][8]: one record per     */
+    int64_t *trace_out;      /* optional DEVICE int64[trace_cap][8] (trace build only:   */
+                             /* lib/libkcore_trace.so; ignored by libkcore.so): one    */
+                             /* record per                                              */
                              /* phase {globaltimer ns, clock64, phase<<8|solo<<4|grid,  */
                              /* k, frontier or scan length, arcs, queue count, 0}       */
     int64_t trace_cap;       /* records available at trace_out (records written are     */

@@ -166,6 +166,9 @@ constexpr int kTraceFields = 8;
 #ifndef KC_BLOOM_GATE
 #define KC_BLOOM_GATE 1  // build the alive-set filter only when the CTA walks >= 1/KC_BLOOM_GATE of the list's length
 #endif
+#ifndef KC_TRACE
+#define KC_TRACE 0  // 1: per-phase / per-CTA trace support (lib/libkcore_trace.so; the checks cost ~2-3 %)
+#endif
 #ifndef KC_SCAN_EC
 #define KC_SCAN_EC 0  // 1 (ablation): level-scan compaction with block scans (Fig. 9) instead of warp ballots
 #endif
@@ -304,6 +307,8 @@ struct Smem {
     Snap snap;
     int32_t qhead, qtail, qpend;
     int32_t near_th1;  // theta + 1 while walks feed a near list, else INT_MIN (set per phase)
+    int64_t *tr_cta;   // per-CTA trace (kcore_options.trace_cta_out) or nullptr, and its capacity
+    int64_t tr_cap;
     unsigned long long qwalked;
     uint32_t bloom[kBloomWords];
 };
@@ -372,22 +377,22 @@ __device__ __forceinline__ bool bloom_maybe(const Smem &sm, uint32_t v)
 // Per-CTA timestamps of the current phase (trace mode only): slot 0 phase
 // start, 1 end of scan / queue walk, 2 end of local drain, 3 barrier arrival.
 // Indexed by the number of grid barriers passed (identical in every CTA).
-__device__ __forceinline__ void cta_time(const KArgs &A, const Ctrl &c, int slot)
+// (the trace pointers are read from shared memory: a global load here would
+// stall thread 0, and with it the CTA's next barrier, on every phase)
+__device__ __forceinline__ void cta_time(const KArgs &A, const Smem &sm, int slot)
 {
-    if (threadIdx.x != 0 || c.solo) return;
-    State *S = A.S;
-    if (!S->trace_cta || c.st_bar >= S->trace_cap) return;
-    S->trace_cta[(c.st_bar * gridDim.x + blockIdx.x) * 8 + slot] = (int64_t)globaltimer();
+    const Ctrl &c = sm.ctrl;
+    if (!KC_TRACE || threadIdx.x != 0 || c.solo || !sm.tr_cta || c.st_bar >= sm.tr_cap) return;
+    sm.tr_cta[(c.st_bar * gridDim.x + blockIdx.x) * 8 + slot] = (int64_t)globaltimer();
 }
 
 // Per-CTA counters of the current phase (trace mode only): slot 4 local
 // sub-rounds, 5 arcs walked, 6 vertices removed, 7 largest sub-round (arcs).
-__device__ __forceinline__ void cta_count(const KArgs &A, const Ctrl &c, int slot, int64_t val)
+__device__ __forceinline__ void cta_count(const KArgs &A, const Smem &sm, int slot, int64_t val)
 {
-    if (threadIdx.x != 0 || c.solo) return;
-    State *S = A.S;
-    if (!S->trace_cta || c.st_bar >= S->trace_cap) return;
-    S->trace_cta[(c.st_bar * gridDim.x + blockIdx.x) * 8 + slot] = val;
+    const Ctrl &c = sm.ctrl;
+    if (!KC_TRACE || threadIdx.x != 0 || c.solo || !sm.tr_cta || c.st_bar >= sm.tr_cap) return;
+    sm.tr_cta[(c.st_bar * gridDim.x + blockIdx.x) * 8 + slot] = val;
 }
 
 // CTA-wide min, then one atomicMin per CTA
@@ -1475,7 +1480,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
 {
     const int wib = threadIdx.x >> 5;
     int lmin = INT_MAX, gcnt = 0;
-    cta_time(A, c, 0);
+    cta_time(A, sm, 0);
 #ifdef KC_PROBE
     if (threadIdx.x == 0) s_probe_k = c.k;
 #endif
@@ -1492,15 +1497,15 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
     __syncthreads();
-    cta_time(A, c, 1);
+    cta_time(A, sm, 1);
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_LOCAL;
     int64_t subs = 0, tmax = 0;
     const int64_t walked = drain(A, sm, c.k, bl, ao, lmin, gcnt, &subs, &tmax);
-    cta_time(A, c, 2);
+    cta_time(A, sm, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
-    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
+    cta_count(A, sm, 4, subs); cta_count(A, sm, 5, walked); cta_count(A, sm, 6, sm.removed); cta_count(A, sm, 7, tmax);
     if (threadIdx.x == 0) {
         const unsigned long long wk = (unsigned long long)walked;
         if (wk) atomicAdd(&A.S->arcs_walked, wk);
@@ -1519,7 +1524,7 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     int64_t C = (T + W - 1) / W;
     C = ((C + kBatch - 1) / kBatch) * kBatch;
     int lmin = INT_MAX, gcnt = 0;
-    cta_time(A, c, 0);
+    cta_time(A, sm, 0);
 #ifdef KC_PROBE
     if (threadIdx.x == 0) s_probe_k = c.k;
 #endif
@@ -1540,9 +1545,9 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
         const int64_t ra0 = c.as + gw * C;
         if (ra0 < c.ae) walk_red(A, sm, c.s, c.e, c.ae, ra0, min(ra0 + C, c.ae), bl);
         __syncthreads();
-        cta_time(A, c, 1);
-        cta_time(A, c, 2);
-        cta_count(A, c, 5, cta_arcs);
+        cta_time(A, sm, 1);
+        cta_time(A, sm, 2);
+        cta_count(A, sm, 5, cta_arcs);
         if (threadIdx.x == 0 && cta_arcs > 0) atomicAdd(&A.S->arcs_walked, (unsigned long long)cta_arcs);
         return;
     }
@@ -1553,13 +1558,13 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
                     gcnt, KC_CF_HUB);
     int64_t walked = cta_arcs;
     __syncthreads();
-    cta_time(A, c, 1);
+    cta_time(A, sm, 1);
     int64_t subs = 0, tmax = 0;
     walked += drain(A, sm, c.k, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
-    cta_time(A, c, 2);
+    cta_time(A, sm, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
-    cta_count(A, c, 4, subs); cta_count(A, c, 5, walked); cta_count(A, c, 6, sm.removed); cta_count(A, c, 7, tmax);
+    cta_count(A, sm, 4, subs); cta_count(A, sm, 5, walked); cta_count(A, sm, 6, sm.removed); cta_count(A, sm, 7, tmax);
     if (threadIdx.x == 0) {
         const unsigned long long wk = (unsigned long long)walked;
         if (wk) atomicAdd(&A.S->arcs_walked, wk);
@@ -1742,7 +1747,7 @@ __device__ __forceinline__ Snap take_snapshot(State *S, unsigned grid, int near_
 
 __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &sn, int grid)
 {
-    if (!S->trace) return;
+    if (!KC_TRACE || !S->trace) return;
     const unsigned long long i = S->trace_n;
     if ((int64_t)i >= S->trace_cap) return;
     int64_t *r = S->trace + i * kTraceFields;
@@ -1763,7 +1768,7 @@ __device__ __forceinline__ void trace_rec(State *S, const Ctrl &c, const Snap &s
 __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
 {
     __syncthreads();
-    cta_time(A, sm.ctrl, 3);
+    cta_time(A, sm, 3);
     if (threadIdx.x == 0) {
         State *S = A.S;
         PROBE(33, 0);
@@ -1844,7 +1849,12 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant_
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
     State *S = A.S;
     const Params p = S->prm;
-    if (threadIdx.x == 0) { init_ctrl(sm.ctrl); sm.ctrl.near_w = p.near_w; }
+    if (threadIdx.x == 0) {
+        init_ctrl(sm.ctrl);
+        sm.ctrl.near_w = p.near_w;
+        sm.tr_cta = S->trace_cta;
+        sm.tr_cap = S->trace_cap;
+    }
 #ifdef KC_PROBE
     if (threadIdx.x == 0) { s_probe_n = 0u; s_probe_k = 0; }
     __syncthreads();
@@ -1901,6 +1911,8 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(const __grid_constant__ KAr
     Smem &sm = *reinterpret_cast<Smem *>(smem_raw);
     if (threadIdx.x == 0) {
         sm.ctrl = A.S->pub;
+        sm.tr_cta = A.S->trace_cta;
+        sm.tr_cap = A.S->trace_cap;
         sm.bloom_on = 0;
         sm.bloom_level = -1;
         sm.seg_cache_ok[0] = sm.seg_cache_ok[1] = 0;

@@ -1,5 +1,8 @@
 """Dump per-phase and per-CTA traces for configs into gpurun_out/ (dev aid)."""
 import sys, os
+# the trace needs the trace build of the library (make builds lib/libkcore_trace.so)
+os.environ.setdefault("KCORE_LIB", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                                                "paper_conf_icde_ahmady0gcz23_b200", "lib", "libkcore_trace.so"))
 import numpy as np
 import torch
 sys.path.insert(0, '.')

@@ -1,7 +1,8 @@
 """Experiment: cost of finishing the peel's tail with MPM on the k*-core
 (dev aid).  For several k*, extract the k*-core (kcore_kcore_subgraph), run
 MPM on it and compare with the peel's time spent on levels >= k* (trace)."""
-import sys
+import os, sys
+os.environ.setdefault("KCORE_LIB", os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "paper_conf_icde_ahmady0gcz23_b200", "lib", "libkcore_trace.so"))
 import numpy as np
 import torch
 sys.path.insert(0, '.')
