@@ -307,6 +307,7 @@ struct Smem {
     Snap snap;
     int32_t qhead, qtail, qpend;
     int32_t near_th1;  // theta + 1 while walks feed a near list, else INT_MIN (set per phase)
+    int32_t bloom_en;  // Params::bloom (kept in shared memory: no global load per phase)
     int64_t *tr_cta;   // per-CTA trace (kcore_options.trace_cta_out) or nullptr, and its capacity
     int64_t tr_cap;
     unsigned long long qwalked;
@@ -1213,7 +1214,7 @@ __device__ void bloom_build(const KArgs &A, const Ctrl &c, Smem &sm)
 // cascade walked by one CTA.
 __device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &sm, int64_t arcs)
 {
-    if (!A.S->prm.bloom) return false;
+    if (!sm.bloom_en) return false;
     const bool have = sm.bloom_on != 0;
     if (have && c.src_len * 2 > sm.bloom_level) return true;
     if (c.src_sel < 0 || c.src_len > kBloomMaxA) return have;
@@ -1854,6 +1855,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant_
         sm.ctrl.near_w = p.near_w;
         sm.tr_cta = S->trace_cta;
         sm.tr_cap = S->trace_cap;
+        sm.bloom_en = p.bloom;
     }
 #ifdef KC_PROBE
     if (threadIdx.x == 0) { s_probe_n = 0u; s_probe_k = 0; }
@@ -1913,6 +1915,7 @@ __global__ void __launch_bounds__(kBlock, 1) k_phase(const __grid_constant__ KAr
         sm.ctrl = A.S->pub;
         sm.tr_cta = A.S->trace_cta;
         sm.tr_cap = A.S->trace_cap;
+        sm.bloom_en = A.S->prm.bloom;
         sm.bloom_on = 0;
         sm.bloom_level = -1;
         sm.seg_cache_ok[0] = sm.seg_cache_ok[1] = 0;
