@@ -1499,13 +1499,16 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
     __syncthreads();
     cta_time(A, sm, 1);
+    if (threadIdx.x == 0) PROBE(40, 0);
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_LOCAL;
     int64_t subs = 0, tmax = 0;
     const int64_t walked = drain(A, sm, c.k, bl, ao, lmin, gcnt, &subs, &tmax);
+    if (threadIdx.x == 0) PROBE(41, 0);
     cta_time(A, sm, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
+    if (threadIdx.x == 0) PROBE(42, 0);
     cta_count(A, sm, 4, subs); cta_count(A, sm, 5, walked); cta_count(A, sm, 6, sm.removed); cta_count(A, sm, 7, tmax);
     if (threadIdx.x == 0) {
         const unsigned long long wk = (unsigned long long)walked;
