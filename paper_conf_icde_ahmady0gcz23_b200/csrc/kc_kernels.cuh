@@ -64,7 +64,7 @@ constexpr int kAsyncNx = 2;          // route target "async chunk queue" (lists 
 // CTA's phase total past kPhase, goes to the global queue (HUB phase) instead
 // of the CTA's own frontier (tuned on B200: DESIGN.md §8).
 #ifndef KC_HUB
-#define KC_HUB 32768
+#define KC_HUB 8192
 #endif
 #ifndef KC_SUB
 #define KC_SUB 32768
@@ -178,6 +178,18 @@ constexpr int kTraceFields = 8;
 #ifndef KC_NEAR
 #define KC_NEAR 1  // 0: compile the near list out (walks never test for theta crossings)
 #endif
+#ifndef KC_ROUTE_FAST
+#define KC_ROUTE_FAST 1  // route_won4: a single claimed vertex per warp takes a short path (C3 -1.5 %, C4 -1 %)
+#endif
+#ifndef KC_PUSH_PAR
+#define KC_PUSH_PAR 1  // async-queue chunks of claimed rows are published by all 32 lanes
+#endif
+#ifndef KC_SPIN_LD
+#define KC_SPIN_LD 0  // (measured: no gain) 1: idle warps of the async drain wait on their slot with plain loads
+#endif
+#ifndef KC_SPIN_NAP
+#define KC_SPIN_NAP 0  // ns of __nanosleep between those polls
+#endif
 enum : int32_t { PH_INIT = 0, PH_LEVEL = 1, PH_HUB = 2, PH_DONE = 3 };
 
 struct Ctrl {
@@ -241,6 +253,7 @@ struct State {
     Snap snap[2];                               // counters at barrier gen, by gen & 1
     alignas(128) unsigned long long arcs_walked;
     alignas(128) unsigned long long near_tail[2];  // near-list append cursors (one line)
+    alignas(128) uint32_t scan_done;            // CTAs whose level scan of this phase is complete
     alignas(128) Ctrl pub;                      // Ctrl published by CTA 0 after a solo run
     alignas(128) Params prm;
     int64_t *trace;                             // optional [trace_cap][kTraceFields]
@@ -308,6 +321,8 @@ struct Smem {
     int32_t qhead, qtail, qpend;
     int32_t near_th1;  // theta + 1 while walks feed a near list, else INT_MIN (set per phase)
     int32_t bloom_en;  // Params::bloom (kept in shared memory: no global load per phase)
+    int32_t nclaim;    // 1: a level scan may still be running somewhere -- hits must claim (see handle_hits)
+    int32_t spec;      // walks load the row bounds of every decremented target with its atomic (KC_SPEC)
     int64_t *tr_cta;   // per-CTA trace (kcore_options.trace_cta_out) or nullptr, and its capacity
     int64_t tr_cap;
     unsigned long long qwalked;
@@ -605,6 +620,51 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
                                         int64_t b0, int64_t b1, int64_t b2, int64_t b3, int nx, int &gcnt)
 {
     const int lane = threadIdx.x & 31;
+#if KC_ROUTE_FAST
+    if (KC_ASYNC && nx == kAsyncNx) {
+        // fast path: ONE vertex claimed by the whole warp (the usual hit of a
+        // light walk) -- no prefix sums, one reservation chain, its chunks
+        // published by all lanes
+        const unsigned anyl = __ballot_sync(kFull, wm != 0u);
+        const int L = __ffs(anyl) - 1;
+        const unsigned wmL = __shfl_sync(kFull, wm, L & 31);
+        if (anyl != 0u && (anyl & (anyl - 1u)) == 0u && (wmL & (wmL - 1u)) == 0u) {
+            const int r = __ffs(wmL) - 1;
+            const int32_t v = __shfl_sync(kFull, r == 0 ? v0 : r == 1 ? v1 : r == 2 ? v2 : v3, L);
+            const int32_t d = __shfl_sync(kFull, r == 0 ? d0 : r == 1 ? d1 : r == 2 ? d2 : d3, L);
+            const int64_t b = __shfl_sync(kFull, r == 0 ? b0 : r == 1 ? b1 : r == 2 ? b2 : b3, L);
+            if (lane == 0) {
+                if (A.order) A.order[atomicAdd(&A.S->ord_tail, 1ULL)] = v;
+                else atomicAdd(&sm.removed, 1);
+            }
+            if (d > 0) {
+                const int nc = (d + kBatch - 1) / kBatch;
+                int ok = 0, base = 0;
+                if (lane == 0 && !KC_NO_SMBUF && d <= sm.bud_hub && atomicAdd(&sm.lphase, d) + d <= sm.bud_phase) {
+                    int t = *(volatile int *)&sm.qtail;
+                    while (t + nc <= kQCap) {
+                        const int o2 = atomicCAS(&sm.qtail, t, t + nc);
+                        if (o2 == t) { ok = 1; base = t; break; }
+                        t = o2;
+                    }
+                    if (ok) atomicAdd(&sm.qpend, nc);  // before any chunk is visible
+                }
+                ok = __shfl_sync(kFull, ok, 0);
+                if (ok) {
+                    base = __shfl_sync(kFull, base, 0);
+                    for (int q = lane; q < nc; q += 32)
+                        atomicExch(&sm.qword[base + q], qword_pack(b + (int64_t)q * kBatch, min(kBatch, d - q * kBatch)));
+                } else {
+                    if (gcnt + 1 > kGStage) gq_flush(A, sm, wib, gcnt);
+                    if (lane == 0) { sm.gv[wib][gcnt] = v; sm.gd[wib][gcnt] = d; sm.gb[wib][gcnt] = b; }
+                    gcnt += 1;
+                }
+            }
+            __syncwarp();
+            return;
+        }
+    }
+#endif
     const unsigned lt = lanemask_lt();
     const int32_t vv[4] = {v0, v1, v2, v3};
     const int32_t dd[4] = {d0, d1, d2, d3};
@@ -628,6 +688,7 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
     } else if (lane == 0) {
         atomicAdd(&sm.removed, tot);
     }
+    if (lane == 0) PROBE_W(15, threadIdx.x >> 5);
     unsigned cm = 0;
 #pragma unroll
     for (int r = 0; r < 4; r++)
@@ -675,15 +736,41 @@ void route_won4(const KArgs &A, Smem &sm, int wib, unsigned wm, int32_t v0, int3
         }
         ok = __shfl_sync(kFull, ok, 0);
         base = __shfl_sync(kFull, base, 0);
+        if (lane == 0) PROBE_W(16, threadIdx.x >> 5);
         if (ok) {
+#if KC_PUSH_PAR
+            // publish the chunks with every lane: a hub row is dozens of chunks,
+            // one lane writing them in sequence stalls the hop by ~1 us
+            int p0[4];
+            p0[0] = base + incl - mine;
+#pragma unroll
+            for (int r = 1; r < 4; r++) p0[r] = p0[r - 1] + nc[r - 1];
+            unsigned any = __ballot_sync(kFull, mine > 0);
+            while (any) {
+                const int L = __ffs(any) - 1;
+                any &= any - 1;
+#pragma unroll
+                for (int r = 0; r < 4; r++) {
+                    const int ncr = __shfl_sync(kFull, nc[r], L);
+                    if (ncr == 0) continue;
+                    const int64_t b = __shfl_sync(kFull, bb[r], L);
+                    const int d = __shfl_sync(kFull, dd[r], L);
+                    const int ps = __shfl_sync(kFull, p0[r], L);
+                    for (int q = lane; q < ncr; q += 32)
+                        atomicExch(&sm.qword[ps + q], qword_pack(b + (int64_t)q * kBatch, min(kBatch, d - q * kBatch)));
+                }
+            }
+#else
             int pos = base + incl - mine;
 #pragma unroll
             for (int r = 0; r < 4; r++) {
                 for (int q = 0; q < nc[r]; q++, pos++)
                     atomicExch(&sm.qword[pos], qword_pack(bb[r] + (int64_t)q * kBatch, min(kBatch, dd[r] - q * kBatch)));
             }
-            lm = cm;
+#endif
+            lm |= cm;
         }
+        if (lane == 0) PROBE_W(17, threadIdx.x >> 5);
     } else if (ctot) {
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) sumd += __shfl_xor_sync(kFull, sumd, o);
@@ -770,14 +857,35 @@ __device__ __forceinline__ void near_push(const KArgs &A, const Smem &sm, int32_
 // --------------------------------------------------------- arc walking
 // Hits of one batch (u reached k): claim, fetch row bounds, prefetch the
 // row's first line for the next hop, route.  Out of line: rare path.
+#ifndef KC_NOCLAIM
+#define KC_NOCLAIM 0  // (C1/C3/C4 ~1 % faster without: the per-batch flag read costs more) 1: hits skip the claim atomic once every level scan of the phase is known complete
+#endif
+#ifndef KC_SPEC
+#define KC_SPEC 0  // (measured slower: extra scattered loads) filtered (light) walks load the row bounds of each decremented target with its atomic
+#endif
+// Hits of one batch (u reached k: old == k+1 from its decrement).  `nc`
+// (read before the batch's decrements): some CTA's level scan of this phase
+// may still be running.  Only a scan can race a hit -- it may read deg[u] <= k
+// after the decrement that took u from k+1 to k -- so while nc, the claim bit
+// decides (atomicOr, reading R9).  Once every scan of the phase has finished
+// before the decrement was issued (scan_done == grid observed, acquire chain:
+// scanner deg read -> red.release -> this CTA's fence -> nclaim store
+// (release.cta) -> walker's acquire.cta load -> its decrement), nothing can
+// race: old == k+1 is seen exactly once, so the hit is owned without a round
+// trip and the claim bit is set fire-and-forget (later scans test it).  HUB
+// phases run no scan at all.  With SPEC the row bounds were loaded together
+// with the decrements (pb0/pb1), so a claim-free hit costs no round trip here.
+template <bool SPEC>
 #if KC_HITS_INLINE
 __device__ __forceinline__
 #else
 __device__ __noinline__
 #endif
 void handle_hits(const KArgs &A, Smem &sm, int k, int nx, int u0, int u1, int u2, int u3,
-                                         unsigned hm, int &gcnt)
+                                         unsigned hm, int &gcnt, bool nc, const int64_t *pb0 = nullptr,
+                                         const int64_t *pb1 = nullptr)
 {
+    const int lane = threadIdx.x & 31;
     const int wib = threadIdx.x >> 5;
     const int uu[4] = {u0, u1, u2, u3};
     // row bounds and claims issued together (independent round trips)
@@ -785,12 +893,33 @@ void handle_hits(const KArgs &A, Smem &sm, int k, int nx, int u0, int u1, int u2
 #pragma unroll
     for (int r = 0; r < 4; r++) {
         const bool h = (hm >> r) & 1u;
-        b0[r] = h ? ld_ro_i64(A.rowptr + uu[r]) : 0;
-        b1[r] = h ? ld_ro_i64(A.rowptr + uu[r] + 1) : 0;
+        if (SPEC) {
+            b0[r] = h ? pb0[r] : 0;
+            b1[r] = h ? pb1[r] : 0;
+        } else {
+            b0[r] = h ? ld_ro_i64(A.rowptr + uu[r]) : 0;
+            b1[r] = h ? ld_ro_i64(A.rowptr + uu[r] + 1) : 0;
+        }
     }
     bool won[4];
+    if (KC_NOCLAIM && !nc) {
 #pragma unroll
-    for (int r = 0; r < 4; r++) won[r] = ((hm >> r) & 1u) && claim(A, uu[r]);
+        for (int r = 0; r < 4; r++) {
+            won[r] = (hm >> r) & 1u;
+            if (won[r]) red_or_u32(A.claimed + (uu[r] >> 5), 1u << (uu[r] & 31));
+        }
+    } else {
+        const unsigned hb = __ballot_sync(kFull, hm != 0);
+        const int lead = __ffs(hb) - 1;
+        uint32_t sd = 0;
+        if (KC_NOCLAIM && lane == lead) sd = ld_relaxed_u32(&A.S->scan_done);  // in flight with the claims
+#pragma unroll
+        for (int r = 0; r < 4; r++) won[r] = ((hm >> r) & 1u) && claim(A, uu[r]);
+        if (KC_NOCLAIM && lane == lead && sd >= gridDim.x) {
+            fence_acq_rel_gpu();
+            st_release_cta_shared(&sm.nclaim, 0);
+        }
+    }
 #ifdef KC_PROBE_W
     {
         int64_t dep = 0;
@@ -911,6 +1040,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
 #pragma unroll
             for (int r = 0; r < kUnroll; r++)
                 d[r] = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
+            const bool nc = __shfl_sync(kFull, ld_acquire_cta_shared(&sm.nclaim), 0) != 0;  // warp-uniform
             int old[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
@@ -924,7 +1054,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             const unsigned hb = __ballot_sync(kFull, hm != 0);
             if (lane == 0) PROBE_W(11, (threadIdx.x >> 5) | ((int64_t)__popc(hb) << 8) | ((int64_t)old[0] << 16));
             if (hb) {
-                handle_hits(A, sm, k, nx, u[0], u[1], u[2], u[3], hm, gcnt);
+                handle_hits<false>(A, sm, k, nx, u[0], u[1], u[2], u[3], hm, gcnt, nc);
             }
             if (lane == 0) PROBE_W(12, threadIdx.x >> 5);
             a = an;
@@ -1095,19 +1225,38 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
 {
     const int lane = threadIdx.x & 31;
     const uint64_t pol = deg_policy();
+    const bool spec = sm.spec != 0;
     int64_t walked = 0;
     while (true) {
         unsigned long long w = 0ULL;
+        int src = 3;  // 1: a chunk, 3: the drain is over
         if (lane == 0) {
+            // blocking ticket: the warp owns slot idx and takes it when published
             const int idx = atomicAdd(&sm.qhead, 1);
             if (idx < kQCap) {
+#if KC_SPIN_LD
+                // wait with plain loads (and a nap): spinning shared-memory
+                // atomics would queue ahead of the working warps' queue updates
+                while (true) {
+                    if (*(volatile unsigned long long *)&sm.qword[idx] != 0ULL) {
+                        w = atomicExch(&sm.qword[idx], 0ULL);  // the slot is this warp's ticket
+                        break;
+                    }
+                    if (*(volatile int *)&sm.qpend == 0) break;
+                    if (KC_SPIN_NAP > 0) __nanosleep(KC_SPIN_NAP);
+                }
+#else
                 while ((w = atomicExch(&sm.qword[idx], 0ULL)) == 0ULL) {
                     if (atomicAdd(&sm.qpend, 0) == 0) break;
                 }
+#endif
+                if (w) src = 1;
             }
         }
         w = __shfl_sync(kFull, w, 0);
-        if (w == 0ULL) break;
+        src = __shfl_sync(kFull, src, 0);
+        if (src == 3) break;
+        if (lane == 0) PROBE_W(20, (threadIdx.x >> 5) | (src << 8));
         const int64_t beg = (int64_t)(w & ((1ULL << 34) - 1ULL));
         const int len = (int)((w >> 34) & 127ULL) + 1;
         int32_t u[kUnroll];
@@ -1121,22 +1270,57 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
             for (int r = 0; r < kUnroll; r++)
                 if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
         }
+#ifdef KC_PROBE_W
+        {
+            const unsigned all = __ballot_sync(kFull, (u[0] ^ u[1] ^ u[2] ^ u[3]) == 7);
+            if (lane == 0) PROBE_W(21, (threadIdx.x >> 5) | ((int64_t)(all & 1u) << 16));
+        }
+#endif
+        const bool nc = __shfl_sync(kFull, ld_acquire_cta_shared(&sm.nclaim), 0) != 0;  // warp-uniform
         int old[kUnroll];
+        if (KC_SPEC && spec) {
+            // light walk: the row bounds of every decremented target travel with
+            // its atomic, so a hit is routed one round trip sooner
+            int64_t sb0[kUnroll], sb1[kUnroll];
 #pragma unroll
-        for (int r = 0; r < kUnroll; r++) {
-            const int32_t d = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
-            old[r] = d > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
-        }
-        unsigned hm = 0;
-        const int th1 = near_th1(sm);
+            for (int r = 0; r < kUnroll; r++) {
+                const bool go = u[r] >= 0;
+                sb0[r] = go ? ld_ro_i64(A.rowptr + u[r]) : 0;
+                sb1[r] = go ? ld_ro_i64(A.rowptr + u[r] + 1) : 0;
+                old[r] = go ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
+            }
+            unsigned hm = 0;
+            const int th1 = near_th1(sm);
 #pragma unroll
-        for (int r = 0; r < kUnroll; r++) {
-            if (old[r] == k + 1) hm |= 1u << r;
-            else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
+            for (int r = 0; r < kUnroll; r++) {
+                if (old[r] == k + 1) hm |= 1u << r;
+                else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
+            }
+            if (__any_sync(kFull, hm != 0))
+                handle_hits<true>(A, sm, k, kAsyncNx, u[0], u[1], u[2], u[3], hm, gcnt, nc, sb0, sb1);
+        } else {
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) {
+                const int32_t d = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
+                old[r] = d > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
+            }
+            unsigned hm = 0;
+            const int th1 = near_th1(sm);
+#pragma unroll
+            for (int r = 0; r < kUnroll; r++) {
+                if (old[r] == k + 1) hm |= 1u << r;
+                else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
+            }
+#ifdef KC_PROBE_W
+            {
+                const unsigned hbp = __ballot_sync(kFull, hm != 0);
+                if (lane == 0) PROBE_W(22, (threadIdx.x >> 5) | ((int64_t)__popc(hbp) << 8) | ((int64_t)old[0] << 16));
+            }
+#endif
+            if (__any_sync(kFull, hm != 0))
+                handle_hits<false>(A, sm, k, kAsyncNx, u[0], u[1], u[2], u[3], hm, gcnt, nc);
         }
-        if (__any_sync(kFull, hm != 0)) {
-            handle_hits(A, sm, k, kAsyncNx, u[0], u[1], u[2], u[3], hm, gcnt);
-        }
+        if (lane == 0) PROBE_W(23, threadIdx.x >> 5);
         walked += len;
         __syncwarp();
         if (lane == 0) atomicSub(&sm.qpend, 1);
@@ -1235,6 +1419,7 @@ __device__ void phase_init(const KArgs &A, Smem &sm)
     const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (threadIdx.x == 0) sm.removed = 0;
     for (int i = threadIdx.x; i < kQCap; i += kBlock) sm.qword[i] = 0ULL;
+
     __syncthreads();
     // The 0-shell is the isolated vertices: nothing can reach them, so
     // they are removed here -- claim bit set, core 0, counted as removed -- and
@@ -1494,6 +1679,7 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.bud_phase = kPhase;
         sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qwalked = 0ULL;
         sm.near_th1 = c.near_app >= 0 ? c.theta + 1 : INT_MIN;
+        sm.nclaim = 1;
     }
     __syncthreads();
     level_scan(A, c, sm, bid, nblk, lmin, gcnt);
@@ -1502,6 +1688,13 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
     if (threadIdx.x == 0) PROBE(40, 0);
     const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
     const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_LOCAL;
+    if (threadIdx.x == 0) {
+        // this CTA's scan is complete (its deg reads happen-before the release)
+        if (nblk == 1) sm.nclaim = 0;  // solo: the only scan was ours
+        else if (KC_NOCLAIM) red_release_add_u32(&A.S->scan_done, 1u);
+        sm.spec = (bl && ao) ? 1 : 0;
+    }
+    // (drain() begins with __syncthreads)
     int64_t subs = 0, tmax = 0;
     const int64_t walked = drain(A, sm, c.k, bl, ao, lmin, gcnt, &subs, &tmax);
     if (threadIdx.x == 0) PROBE(41, 0);
@@ -1545,6 +1738,11 @@ __device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int 
     __syncthreads();
     const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
     const bool bl = want_bloom(A, c, sm, cta_arcs);
+    if (threadIdx.x == 0) {
+        sm.nclaim = 0;  // a HUB phase runs no scan: nothing races its hits
+        sm.spec = (bl && (bl || KC_AO_ALWAYS) && KC_AO_HUB) ? 1 : 0;
+    }
+    __syncthreads();
     if (c.red) {  // non-returning walk; the next phase rescans (advance())
         const int64_t ra0 = c.as + gw * C;
         if (ra0 < c.ae) walk_red(A, sm, c.s, c.e, c.ae, ra0, min(ra0 + C, c.ae), bl);
@@ -1625,7 +1823,7 @@ __device__ __forceinline__ void setup_near(Ctrl &c, const Snap &sn, const Params
     c.src_single = c.alive_single;
     c.src_len = c.alive_sel < 0 ? p.n : c.alive_len;
     c.compact = 0;
-    c.solo = 0;
+    c.solo = 0;  // (solo near levels on CTA 0 measured 3-15 % slower: one SM's atomic rate)
     c.near_app = c.near_cur ^ 1;
     c.near_reset = c.near_cur;
     if (c.near_lv == 0) c.near_first = c.near_len;
@@ -1742,6 +1940,7 @@ __device__ __forceinline__ Snap take_snapshot(State *S, unsigned grid, int near_
     sn.pad = 0;
     S->alive_out = 0ULL;
     S->min_next = INT_MAX;
+    S->scan_done = 0u;
     // the list this phase consumed (a near scan's source / the previous list of
     // a build) is empty from now on; nobody appends to it until it is a scan's
     // destination again
@@ -1964,6 +2163,7 @@ __global__ void k_init_state(State *S, int64_t n, int32_t solo_arcs, int32_t sol
         S->bar_gen = 0u;
         S->arcs_walked = 0ULL;
         S->near_tail[0] = S->near_tail[1] = 0ULL;
+        S->scan_done = 0u;
         Ctrl z;
         init_ctrl(z);
         z.near_w = near_w > 0 ? near_w : KC_NEAR_W;

@@ -101,8 +101,11 @@ size_t carve(void *base, int64_t n, Carve *c)
     // segments of ceil(n/grid) + 32 entries (the identity scan's slices are 32-aligned)
     t.alive0 = (int32_t *)take(sizeof(int32_t) * (nn + 33 * (size_t)kMaxSeg));
     t.alive1 = (int32_t *)take(sizeof(int32_t) * (nn + 33 * (size_t)kMaxSeg));
-    t.near0 = (int32_t *)take(sizeof(int32_t) * nn);
-    t.near1 = (int32_t *)take(sizeof(int32_t) * nn);
+    // near lists: 2n entries -- a vertex appears at most twice per epoch (the
+    // build's scan may collect it after a walk already appended its theta+1 ->
+    // theta crossing; near scans copy both entries, their claims dedup)
+    t.near0 = (int32_t *)take(sizeof(int32_t) * 2 * nn);
+    t.near1 = (int32_t *)take(sizeof(int32_t) * 2 * nn);
     t.seg0 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     t.seg1 = (int32_t *)take(sizeof(int32_t) * kMaxSeg);
     // claim bits and working degrees adjacent: one L2 access-policy window

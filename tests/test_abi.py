@@ -50,7 +50,7 @@ def test_strerror_and_version():
 def test_workspace_size_scales_linearly():
     a = kc.kcore_workspace_size(1 << 20, 1 << 24)
     b = kc.kcore_workspace_size(1 << 21, 1 << 24)
-    assert 26 * (1 << 20) <= a <= 48 * (1 << 20) + (8 << 20)  # ~44 n B (queues, alive + near lists, bits, degrees) + segment slack
+    assert 26 * (1 << 20) <= a <= 56 * (1 << 20) + (8 << 20)  # ~52 n B (queues, alive + near lists, bits, degrees) + segment slack
     assert b > a
 
 

@@ -3,7 +3,7 @@
 import sys
 import numpy as np
 P = np.load(sys.argv[1])["p"].astype(np.int64)
-names = {20: "pop", 21: "colidx", 22: "atomics", 14: "claims", 23: "routed", 30: "phase", 33: "arrive"}
+names = {20: "pop", 21: "colidx", 22: "atomics", 14: "claims", 15: "r_removed", 16: "r_reserved", 17: "r_pushed", 23: "routed", 30: "phase", 33: "arrive"}
 d = {}
 for cta in np.unique(P[:, 0]):
     Q = P[P[:, 0] == cta]
@@ -12,7 +12,7 @@ for cta in np.unique(P[:, 0]):
     for _, tag, t, val in Q:
         if tag not in names:
             continue
-        w = val & 0xff if tag in (20, 21, 22, 14, 23) else -1
+        w = val & 0xff if tag in (20, 21, 22, 14, 15, 16, 17, 23) else -1
         if tag in (30, 33):
             last = {}
             continue
