@@ -1040,7 +1040,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
 #pragma unroll
             for (int r = 0; r < kUnroll; r++)
                 d[r] = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
-            const bool nc = __shfl_sync(kFull, ld_acquire_cta_shared(&sm.nclaim), 0) != 0;  // warp-uniform
+            const bool nc = !KC_NOCLAIM || __shfl_sync(kFull, ld_acquire_cta_shared(&sm.nclaim), 0) != 0;  // warp-uniform
             int old[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
@@ -1276,7 +1276,7 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
             if (lane == 0) PROBE_W(21, (threadIdx.x >> 5) | ((int64_t)(all & 1u) << 16));
         }
 #endif
-        const bool nc = __shfl_sync(kFull, ld_acquire_cta_shared(&sm.nclaim), 0) != 0;  // warp-uniform
+        const bool nc = !KC_NOCLAIM || __shfl_sync(kFull, ld_acquire_cta_shared(&sm.nclaim), 0) != 0;  // warp-uniform
         int old[kUnroll];
         if (KC_SPEC && spec) {
             // light walk: the row bounds of every decremented target travel with
@@ -1617,38 +1617,43 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
         ndst = A.near[c.near_cur ^ 1];
         ntail = &A.S->near_tail[c.near_cur ^ 1];
     }
-    if (c.near_scan) {  // the near list: one contiguous run, an even slice per CTA, no alive compaction
-        const int64_t L = c.near_len;
-        const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
-        scan_range<false>(A, c, sm, A.near[c.near_cur], lo, hi, nullptr, lmin, gcnt, ndst, ntail);
-        __syncthreads();
-        return;
-    }
     const int32_t *srcb = c.src_sel < 0 ? nullptr : A.alive[c.src_sel];
-    int32_t *dstb = c.compact ? A.alive[c.dst_sel] : nullptr;
+    int32_t *dstb = c.compact ? A.alive[c.dst_sel] : nullptr;  // (a near scan never compacts the alive list)
     const int dseg = solo ? 0 : bid;
     if (threadIdx.x == 0) sm.kcur = 0;
     __syncthreads();
     int32_t *dst = dstb ? dstb + (int64_t)dseg * A.seg_R : nullptr;
-    if (c.src_sel < 0 || c.src_single) {
-        // contiguous source of c.src_len entries: an even slice per CTA
+    if (!c.near_scan && c.src_sel < 0) {
+        // the identity: 32-aligned slices (one claim-bit word per warp item)
         const int64_t L = c.src_len;
-        if (c.src_sel < 0) {  // the identity: 32-aligned slices (one claim-bit word per warp item)
-            const int64_t W = (L + 31) / 32;
-            const int64_t lo = solo ? 0 : 32 * ((W * bid) / nblk), hi = solo ? L : min(L, 32 * ((W * (bid + 1)) / nblk));
-            scan_range<true>(A, c, sm, nullptr, lo, hi, dst, lmin, gcnt, ndst, ntail);
-        } else {
-            const int64_t lo = solo ? 0 : (L * bid) / nblk, hi = solo ? L : (L * (bid + 1)) / nblk;
-            scan_range<false>(A, c, sm, srcb, lo, hi, dst, lmin, gcnt, ndst, ntail);
-        }
-    } else if (!solo) {
-        // this CTA wrote its own segment's length at the last compaction
-        const int64_t len = sm.seg_cache_ok[c.src_sel] ? sm.seg_cache[c.src_sel] : ld_cg_i32(A.seg_len[c.src_sel] + bid);
-        scan_range<false>(A, c, sm, srcb + (int64_t)bid * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
+        const int64_t W = (L + 31) / 32;
+        const int64_t lo = solo ? 0 : 32 * ((W * bid) / nblk), hi = solo ? L : min(L, 32 * ((W * (bid + 1)) / nblk));
+        scan_range<true>(A, c, sm, nullptr, lo, hi, dst, lmin, gcnt, ndst, ntail);
     } else {
-        for (int b = 0; b < A.nseg; b++) {
-            const int64_t len = ld_cg_i32(A.seg_len[c.src_sel] + b);
-            if (len) scan_range<false>(A, c, sm, srcb + (int64_t)b * A.seg_R, 0, len, dst, lmin, gcnt, ndst, ntail);
+        // one call site for every list layout (each inlined copy of scan_range
+        // grows the kernel): the near list or a contiguous alive list -- an even
+        // slice per CTA; per-CTA segments -- this CTA's own, or all of them (solo)
+        const bool segs = !c.near_scan && !c.src_single;
+        const int nit = (segs && solo) ? A.nseg : 1;
+        for (int it = 0; it < nit; it++) {
+            const int32_t *src;
+            int64_t lo, hi;
+            if (!segs) {
+                src = c.near_scan ? A.near[c.near_cur] : srcb;
+                const int64_t L = c.near_scan ? c.near_len : c.src_len;
+                lo = solo ? 0 : (L * bid) / nblk;
+                hi = solo ? L : (L * (bid + 1)) / nblk;
+            } else if (!solo) {
+                // this CTA wrote its own segment's length at the last compaction
+                src = srcb + (int64_t)bid * A.seg_R;
+                lo = 0;
+                hi = sm.seg_cache_ok[c.src_sel] ? sm.seg_cache[c.src_sel] : ld_cg_i32(A.seg_len[c.src_sel] + bid);
+            } else {
+                src = srcb + (int64_t)it * A.seg_R;
+                lo = 0;
+                hi = ld_cg_i32(A.seg_len[c.src_sel] + it);
+            }
+            scan_range<false>(A, c, sm, src, lo, hi, dst, lmin, gcnt, ndst, ntail);
         }
     }
     __syncthreads();
@@ -1660,11 +1665,15 @@ __device__ void level_scan(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int
     }
 }
 
-// One level (Alg. 1 round k): scan this CTA's segment(s), then drain the
-// local frontier breadth-first.
-__device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
+// One phase.  LEVEL (Alg. 1 round k): scan this CTA's segment(s), then drain
+// the local frontier breadth-first.  HUB: walk this CTA's even share of the
+// global queue's arcs (non-returning when c.red), then drain what it claimed.
+// LEVEL and HUB share ONE drain call site (each inlined copy of the drain
+// machinery grows the kernel; measured: a larger kernel runs slower).
+__device__ void run_phase(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
 {
     const int wib = threadIdx.x >> 5;
+    const bool hub = c.phase == PH_HUB;
     int lmin = INT_MAX, gcnt = 0;
     cta_time(A, sm, 0);
 #ifdef KC_PROBE
@@ -1679,93 +1688,57 @@ __device__ void phase_level(const KArgs &A, const Ctrl &c, Smem &sm, int bid, in
         sm.bud_phase = kPhase;
         sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qwalked = 0ULL;
         sm.near_th1 = c.near_app >= 0 ? c.theta + 1 : INT_MIN;
-        sm.nclaim = 1;
+        sm.nclaim = hub ? 0 : 1;  // a HUB phase runs no scan: nothing races its hits
     }
     __syncthreads();
-    level_scan(A, c, sm, bid, nblk, lmin, gcnt);
-    __syncthreads();
-    cta_time(A, sm, 1);
-    if (threadIdx.x == 0) PROBE(40, 0);
-    const bool bl = want_bloom(A, c, sm, (int64_t)sm.larc[0]);
-    const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_LOCAL;
+    // HUB: this CTA's share of the queue's arcs
+    const int64_t gw = (int64_t)bid * kWarps + wib;
+    const int64_t W = (int64_t)nblk * kWarps;
+    int64_t C = (c.ae - c.as + W - 1) / W;
+    C = ((C + kBatch - 1) / kBatch) * kBatch;
+    const int64_t cta_arcs =
+        hub ? min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C) : 0;
+    if (!hub) {
+        level_scan(A, c, sm, bid, nblk, lmin, gcnt);
+        __syncthreads();
+        cta_time(A, sm, 1);
+        if (threadIdx.x == 0) PROBE(40, 0);
+    }
+    const bool bl = want_bloom(A, c, sm, hub ? cta_arcs : (int64_t)sm.larc[0]);
+    const bool ao = (bl || KC_AO_ALWAYS) && (hub ? KC_AO_HUB : KC_AO_LOCAL);
     if (threadIdx.x == 0) {
-        // this CTA's scan is complete (its deg reads happen-before the release)
-        if (nblk == 1) sm.nclaim = 0;  // solo: the only scan was ours
-        else if (KC_NOCLAIM) red_release_add_u32(&A.S->scan_done, 1u);
+        // (LEVEL) this CTA's scan is complete (its deg reads happen-before the release)
+        if (!hub && nblk == 1) sm.nclaim = 0;  // solo: the only scan was ours
+        else if (!hub && KC_NOCLAIM) red_release_add_u32(&A.S->scan_done, 1u);
         sm.spec = (bl && ao) ? 1 : 0;
+    }
+    int64_t walked = cta_arcs;
+    if (hub) {
+        __syncthreads();
+        const int64_t a0 = c.as + gw * C;
+        if (c.red) {  // non-returning walk; the next phase rescans (advance())
+            if (a0 < c.ae) walk_red(A, sm, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl);
+            __syncthreads();
+            cta_time(A, sm, 1);
+            cta_time(A, sm, 2);
+            cta_count(A, sm, 5, cta_arcs);
+            if (threadIdx.x == 0 && cta_arcs > 0) atomicAdd(&A.S->arcs_walked, (unsigned long long)cta_arcs);
+            return;
+        }
+        if (a0 < c.ae)
+            walk<false>(A, sm, c.k, 0, KC_ASYNC == 1 ? kAsyncNx : 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao,
+                        lmin, gcnt, KC_CF_HUB);
+        __syncthreads();
+        cta_time(A, sm, 1);
     }
     // (drain() begins with __syncthreads)
     int64_t subs = 0, tmax = 0;
-    const int64_t walked = drain(A, sm, c.k, bl, ao, lmin, gcnt, &subs, &tmax);
+    walked += drain(A, sm, c.k, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
     if (threadIdx.x == 0) PROBE(41, 0);
     cta_time(A, sm, 2);
     gq_flush(A, sm, wib, gcnt);
     __syncthreads();
     if (threadIdx.x == 0) PROBE(42, 0);
-    cta_count(A, sm, 4, subs); cta_count(A, sm, 5, walked); cta_count(A, sm, 6, sm.removed); cta_count(A, sm, 7, tmax);
-    if (threadIdx.x == 0) {
-        const unsigned long long wk = (unsigned long long)walked;
-        if (wk) atomicAdd(&A.S->arcs_walked, wk);
-        if (sm.removed) atomicAdd(&A.S->ord_tail, (unsigned long long)sm.removed);
-    }
-    block_min_atomic(sm, lmin, &A.S->min_next);
-}
-
-// -------------------------------------------------------------------- HUB
-__device__ void phase_hub(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
-{
-    const int wib = threadIdx.x >> 5;
-    const int64_t gw = (int64_t)bid * kWarps + wib;
-    const int64_t W = (int64_t)nblk * kWarps;
-    const int64_t T = c.ae - c.as;
-    int64_t C = (T + W - 1) / W;
-    C = ((C + kBatch - 1) / kBatch) * kBatch;
-    int lmin = INT_MAX, gcnt = 0;
-    cta_time(A, sm, 0);
-#ifdef KC_PROBE
-    if (threadIdx.x == 0) s_probe_k = c.k;
-#endif
-    if (threadIdx.x == 0) PROBE(30, c.k * 4 + c.phase);
-    if (threadIdx.x == 0) {
-        sm.lcnt[0] = sm.lcnt[1] = 0; sm.larc[0] = sm.larc[1] = 0;
-        sm.lphase = 0; sm.removed = 0;
-        sm.bud_hub = kHub;
-        sm.bud_sub = kSub;
-        sm.bud_phase = kPhase;
-        sm.qhead = 0; sm.qtail = 0; sm.qpend = 0; sm.qwalked = 0ULL;
-        sm.near_th1 = c.near_app >= 0 ? c.theta + 1 : INT_MIN;
-    }
-    __syncthreads();
-    const int64_t cta_arcs = min(c.ae, c.as + (int64_t)(bid + 1) * kWarps * C) - min(c.ae, c.as + (int64_t)bid * kWarps * C);
-    const bool bl = want_bloom(A, c, sm, cta_arcs);
-    if (threadIdx.x == 0) {
-        sm.nclaim = 0;  // a HUB phase runs no scan: nothing races its hits
-        sm.spec = (bl && (bl || KC_AO_ALWAYS) && KC_AO_HUB) ? 1 : 0;
-    }
-    __syncthreads();
-    if (c.red) {  // non-returning walk; the next phase rescans (advance())
-        const int64_t ra0 = c.as + gw * C;
-        if (ra0 < c.ae) walk_red(A, sm, c.s, c.e, c.ae, ra0, min(ra0 + C, c.ae), bl);
-        __syncthreads();
-        cta_time(A, sm, 1);
-        cta_time(A, sm, 2);
-        cta_count(A, sm, 5, cta_arcs);
-        if (threadIdx.x == 0 && cta_arcs > 0) atomicAdd(&A.S->arcs_walked, (unsigned long long)cta_arcs);
-        return;
-    }
-    const bool ao = (bl || KC_AO_ALWAYS) && KC_AO_HUB;
-    const int64_t a0 = c.as + gw * C;
-    if (a0 < c.ae)
-        walk<false>(A, sm, c.k, 0, KC_ASYNC == 1 ? kAsyncNx : 0, c.s, c.e, c.ae, a0, min(a0 + C, c.ae), bl, ao, lmin,
-                    gcnt, KC_CF_HUB);
-    int64_t walked = cta_arcs;
-    __syncthreads();
-    cta_time(A, sm, 1);
-    int64_t subs = 0, tmax = 0;
-    walked += drain(A, sm, c.k, bl, ao && KC_AO_LOCAL, lmin, gcnt, &subs, &tmax);
-    cta_time(A, sm, 2);
-    gq_flush(A, sm, wib, gcnt);
-    __syncthreads();
     cta_count(A, sm, 4, subs); cta_count(A, sm, 5, walked); cta_count(A, sm, 6, sm.removed); cta_count(A, sm, 7, tmax);
     if (threadIdx.x == 0) {
         const unsigned long long wk = (unsigned long long)walked;
@@ -2006,33 +1979,6 @@ __device__ __forceinline__ void grid_barrier(const KArgs &A, Smem &sm)
     __syncthreads();
 }
 
-__device__ __forceinline__ void run_phase(const KArgs &A, const Ctrl &c, Smem &sm, int bid, int nblk)
-{
-    if (c.phase == PH_LEVEL) phase_level(A, c, sm, bid, nblk);
-    else if (c.phase == PH_HUB) phase_hub(A, c, sm, bid, nblk);
-}
-
-// CTA 0 alone: run consecutive solo phases with CTA-local synchronisation.
-__device__ void solo_run(const KArgs &A, Smem &sm, const Params &p)
-{
-    State *S = A.S;
-    while (true) {
-        const Ctrl &c = sm.ctrl;  // shared copy: no per-thread spill
-        run_phase(A, c, sm, 0, 1);  // ends with __syncthreads (block_min_atomic)
-        if (threadIdx.x == 0) {
-            __threadfence();
-            const Snap sn = take_snapshot(S, 1u, sm.ctrl.near_reset);
-            trace_rec(S, sm.ctrl, sn, 0);
-            advance(sm.ctrl, sn, p);
-        }
-        __syncthreads();
-        if (sm.ctrl.phase == PH_DONE || !sm.ctrl.solo) break;
-    }
-    if (threadIdx.x == 0) {
-        S->pub = sm.ctrl;
-        __threadfence();
-    }
-}
 
 __device__ __forceinline__ void init_ctrl(Ctrl &z)
 {
@@ -2069,8 +2015,29 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant_
     __syncthreads();
     while (true) {
         if (sm.ctrl.phase == PH_DONE) break;
-        if (sm.ctrl.solo) {
-            if (blockIdx.x == 0) solo_run(A, sm, p);
+        // ONE call site of the phase code (a second one -- e.g. a separate solo
+        // loop -- duplicates every inlined phase function: measured, the larger
+        // kernel runs slower even where the copy is never executed)
+        const bool solo = sm.ctrl.solo != 0;
+        if (threadIdx.x == 0 && !solo) PROBE(38, 0);
+        if (!solo || blockIdx.x == 0) run_phase(A, sm.ctrl, sm, solo ? 0 : blockIdx.x, solo ? 1 : gridDim.x);
+        if (solo) {
+            // CTA 0 alone, CTA-local synchronisation: consecutive solo phases
+            // run without a grid barrier; the others wait at the next one
+            if (blockIdx.x == 0) {
+                if (threadIdx.x == 0) {
+                    __threadfence();
+                    const Snap sn = take_snapshot(S, 1u, sm.ctrl.near_reset);
+                    trace_rec(S, sm.ctrl, sn, 0);
+                    advance(sm.ctrl, sn, p);
+                }
+                __syncthreads();
+                if (sm.ctrl.phase != PH_DONE && sm.ctrl.solo) continue;
+                if (threadIdx.x == 0) {
+                    S->pub = sm.ctrl;
+                    __threadfence();
+                }
+            }
             grid_barrier(A, sm);
             if (threadIdx.x == 0) {
                 Ctrl c;
@@ -2082,9 +2049,6 @@ __global__ void __launch_bounds__(kBlock, 1) k_persistent(const __grid_constant_
                 sm.ctrl = c;
             }
         } else {
-            if (threadIdx.x == 0) PROBE(38, 0);
-            const Ctrl &c = sm.ctrl;  // shared copy: no per-thread spill
-            run_phase(A, c, sm, blockIdx.x, gridDim.x);
             grid_barrier(A, sm);
             if (threadIdx.x == 0) {
                 PROBE(36, 0);
