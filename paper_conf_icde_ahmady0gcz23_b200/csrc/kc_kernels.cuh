@@ -1506,8 +1506,22 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
             // in a lazily compacted list fail the claim.  At k = 0 the frontier
             // is the isolated vertices: nothing walks, nothing races.
             if (vv[j] < 0) continue;
-            if (dd[j] <= k) { if (IDENT || k == 0 || claim(A, vv[j])) wm |= 1u << j; }
-            else if (dd[j] > k) { lmin = min(lmin, dd[j]); km |= 1u << j; }
+            if (dd[j] <= k) wm |= 1u << j;
+            else { lmin = min(lmin, dd[j]); km |= 1u << j; }
+        }
+        // row bounds of every candidate, in flight together with its claim
+        // (at k = 0 every candidate is isolated)
+        int64_t b0[kScanItems], e0[kScanItems];
+#pragma unroll
+        for (int j = 0; j < kScanItems; j++) {
+            const bool cand = ((wm >> j) & 1u) && k > 0;
+            b0[j] = cand ? ld_ro_i64(A.rowptr + vv[j]) : 0;
+            e0[j] = cand ? ld_ro_i64(A.rowptr + vv[j] + 1) : 0;
+        }
+        if (!IDENT && k > 0) {
+#pragma unroll
+            for (int j = 0; j < kScanItems; j++)
+                if (((wm >> j) & 1u) && !claim(A, vv[j])) wm &= ~(1u << j);
         }
         if (IDENT && k > 0) {
             // identity scan (ids lo..hi-1, the first level): the 32 lanes of item j
@@ -1578,17 +1592,9 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
         for (int j = 0; j < kScanItems; j++)
             if ((wm >> j) & 1u) A.core[vv[j]] = k;
         if (__any_sync(kFull, wm != 0)) {
-            // row bounds of every claimed vertex first (all loads in flight), then route
-            int64_t b0[kScanItems];
             int32_t du[kScanItems];
 #pragma unroll
-            for (int j = 0; j < kScanItems; j++) {
-                b0[j] = 0; du[j] = 0;
-                if (((wm >> j) & 1u) && k > 0) {  // at k = 0 every claimed vertex is isolated
-                    b0[j] = ld_ro_i64(A.rowptr + vv[j]);
-                    du[j] = (int32_t)(ld_ro_i64(A.rowptr + vv[j] + 1) - b0[j]);
-                }
-            }
+            for (int j = 0; j < kScanItems; j++) du[j] = ((wm >> j) & 1u) ? (int32_t)(e0[j] - b0[j]) : 0;
 #pragma unroll
             for (int j = 0; j < kScanItems; j++)
                 if (du[j] > 0) prefetch_row(A.colidx, b0[j], b0[j] + du[j]);
