@@ -501,7 +501,7 @@ __device__ __forceinline__
 #else
 __device__ __noinline__
 #endif
-void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
+void gq_flush_(const KArgs &A, Smem &sm, int wib, int gcnt)
 {
     const int lane = threadIdx.x & 31;
     if (gcnt == 0) return;
@@ -532,6 +532,13 @@ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
         carry += __shfl_sync(kFull, incl, 31);
     }
     __syncwarp();
+}
+
+// (gcnt passed by value: a reference across the out-of-line call kept the
+// stage count in local memory on every routing path)
+__device__ __forceinline__ void gq_flush(const KArgs &A, Smem &sm, int wib, int &gcnt)
+{
+    if (gcnt) gq_flush_(A, sm, wib, gcnt);
     gcnt = 0;
 }
 
