@@ -23,3 +23,8 @@ ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-fil
     python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-mpm --no-configs > $O/launches.log 2>&1
 python tools/cta_trace.py fin C1 C2 C3 C4 > $O/trace.log 2>&1
 python tools/phase_breakdown.py fin C1 C2 C3 C4 > $O/phase_breakdown.json 2> $O/phase_breakdown.err
+if [ -n "$FULL" ]; then
+  # the paper's Table II variants (build them first: bash tools/build_variants.sh tools/variants_f4.txt)
+  python tools/ablation_r2.py > $O/ablation_r2.json 2> $O/ablation.err
+  python tools/c5_run.py > $O/c5.log 2>&1; cp gpurun_out/c5.json $O/c5_r2.json 2>/dev/null
+fi
