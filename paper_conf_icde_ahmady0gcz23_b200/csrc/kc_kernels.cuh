@@ -163,6 +163,9 @@ constexpr int kTraceFields = 8;
 #ifndef KC_NEAR_W
 #define KC_NEAR_W 16
 #endif
+#ifndef KC_BLOOM_MULT
+#define KC_BLOOM_MULT 1  // ... and only when it walks >= KC_BLOOM_MULT x the list's length
+#endif
 #ifndef KC_BLOOM_GATE
 #define KC_BLOOM_GATE 1  // build the alive-set filter only when the CTA walks >= 1/KC_BLOOM_GATE of the list's length
 #endif
@@ -1411,7 +1414,7 @@ __device__ __forceinline__ bool want_bloom(const KArgs &A, const Ctrl &c, Smem &
     if (c.src_sel < 0 || c.src_len > kBloomMaxA) return have;
     // building costs one pass over the alive list per CTA: only for a walk
     // of comparable size (CTA-uniform: arcs is this CTA's pending walk)
-    if (KC_BLOOM_GATE > 0 && arcs * KC_BLOOM_GATE < c.src_len) return have;
+    if (KC_BLOOM_GATE > 0 && arcs * KC_BLOOM_GATE < c.src_len * KC_BLOOM_MULT) return have;
     bloom_build(A, c, sm);
     return true;
 }
