@@ -163,6 +163,12 @@ constexpr int kTraceFields = 8;
 #ifndef KC_NEAR_W
 #define KC_NEAR_W 16
 #endif
+#ifndef KC_PRED_ATOM
+#define KC_PRED_ATOM 1
+#endif
+#ifndef KC_BLOOM_BF
+#define KC_BLOOM_BF 1  // Bloom probes without per-arc branches (C3 -0.9 %)
+#endif
 #ifndef KC_BLOOM_MULT
 #define KC_BLOOM_MULT 1  // ... and only when it walks >= KC_BLOOM_MULT x the list's length
 #endif
@@ -861,6 +867,21 @@ __device__ __forceinline__ void near_push(const KArgs &A, const Smem &sm, int32_
     A.near[app][pos] = u;
 }
 
+// old = atomicSub(p, 1) if go, else INT_MIN -- as ONE predicated atomic
+// (KC_PRED_ATOM; the ternary compiles to a branch + reconvergence per arc)
+__device__ __forceinline__ int atom_dec_if(bool go, int32_t *p, uint64_t pol)
+{
+#if KC_PRED_ATOM && !KC_DEG_EVICT_LAST
+    (void)pol;
+    int old = INT_MIN;
+    asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %2, 0;\n\t@q atom.global.add.s32 %0, [%1], -1;\n\t}"
+                 : "+r"(old) : "l"(p), "r"((unsigned)go) : "memory");
+    return old;
+#else
+    return go ? atom_dec_deg(p, pol) : INT_MIN;
+#endif
+}
+
 // Near list: targets whose decrement crossed theta+1 -> theta (cm bit r set for
 // u[r]) join near[near_app] -- one warp-aggregated append.  Each vertex crosses
 // once per epoch (degrees only decrease), so the list stays within n.
@@ -1032,7 +1053,15 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             if (use_bloom) {
 #pragma unroll
                 for (int r = 0; r < kUnroll; r++)
+                    {
+#if KC_BLOOM_BF
+                    // branch-free: both probes for every lane (a -1 id probes harmlessly)
+                    const bool keep = bloom_maybe(sm, (uint32_t)u[r]);
+                    u[r] = keep ? u[r] : -1;
+#else
                     if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
+#endif
+                }
             }
             if (claim_filter) {
                 // exact dead-target filter: the claim bitmap (2 MB at C4, L1/L2
@@ -1053,7 +1082,7 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             const bool nc = !KC_NOCLAIM || __shfl_sync(kFull, ld_acquire_cta_shared(&sm.nclaim), 0) != 0;  // warp-uniform
             int old[kUnroll];
 #pragma unroll
-            for (int r = 0; r < kUnroll; r++) old[r] = d[r] > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
+            for (int r = 0; r < kUnroll; r++) old[r] = atom_dec_if(d[r] > k, A.deg + u[r], pol);
             unsigned hm = 0;
             const int th1 = near_th1(sm);
 #pragma unroll
@@ -1278,7 +1307,15 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
         if (use_bloom) {
 #pragma unroll
             for (int r = 0; r < kUnroll; r++)
-                if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
+                {
+#if KC_BLOOM_BF
+                    // branch-free: both probes for every lane (a -1 id probes harmlessly)
+                    const bool keep = bloom_maybe(sm, (uint32_t)u[r]);
+                    u[r] = keep ? u[r] : -1;
+#else
+                    if (u[r] >= 0 && !bloom_maybe(sm, (uint32_t)u[r])) u[r] = -1;
+#endif
+                }
         }
 #ifdef KC_PROBE_W
         {
@@ -1312,7 +1349,7 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
                 const int32_t d = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
-                old[r] = d > k ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
+                old[r] = atom_dec_if(d > k, A.deg + u[r], pol);
             }
             unsigned hm = 0;
             const int th1 = near_th1(sm);
