@@ -1186,7 +1186,14 @@ __device__ void walk_red(const KArgs &A, Smem &sm, int64_t s, int64_t e, int64_t
             if (an < limit) gather(an, un);
 #pragma unroll
             for (int r = 0; r < U; r++) {
+#if KC_PRED_ATOM
+                // branch-free: the filter result predicates the red
+                const bool go = u[r] >= 0 && (!use_bloom || bloom_maybe(sm, (uint32_t)u[r]));
+                asm volatile("{\n\t.reg .pred q;\n\tsetp.ne.u32 q, %1, 0;\n\t@q red.global.add.s32 [%0], -1;\n\t}"
+                             ::"l"(A.deg + u[r]), "r"((unsigned)go) : "memory");
+#else
                 if (u[r] >= 0 && (!use_bloom || bloom_maybe(sm, (uint32_t)u[r]))) red_dec(A.deg + u[r]);
+#endif
             }
             a = an;
         }
