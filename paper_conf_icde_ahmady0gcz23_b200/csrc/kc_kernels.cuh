@@ -163,6 +163,12 @@ constexpr int kTraceFields = 8;
 #ifndef KC_NEAR_W
 #define KC_NEAR_W 16
 #endif
+#ifndef KC_WALK_FAST
+#define KC_WALK_FAST 1  // walk<>: a batch inside one row skips the per-arc entry search
+#endif
+#ifndef KC_HIT_BF
+#define KC_HIT_BF 1  // decrement outcomes (hit mask, level-skip min) without per-arc branches
+#endif
 #ifndef KC_PRED_ATOM
 #define KC_PRED_ATOM 1
 #endif
@@ -1027,6 +1033,21 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             const int64_t rq = wq - ab;
             const int32_t q32 = rq < -1 ? -1 : (rq > 0x7fffffff ? 0x7fffffff : (int32_t)rq);
             const int32_t lim = (int32_t)min((int64_t)kBatch, limit - ab);
+#if KC_WALK_FAST
+            // fast path: the whole batch lies in one entry (a long row) -- no search
+            const unsigned le = __ballot_sync(kFull, q32 <= 0);
+            const int first = le ? 31 - __clz(le) : 0;
+            const int32_t qn = __shfl_sync(kFull, q32, min(first + 1, 31));
+            if (first == 31 || qn >= kBatch) {
+                const int64_t off = __shfl_sync(kFull, bmq, first) + ab;
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++) {
+                    const int32_t my = r * 32 + lane;
+                    out[r] = (my < lim) ? ld_stream_i32(A.colidx + off + my) : -1;
+                }
+                return;
+            }
+#endif
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
                 const int32_t my = r * 32 + lane;
@@ -1083,13 +1104,27 @@ __device__ __forceinline__ void walk(const KArgs &A, Smem &sm, const int k, cons
             int old[kUnroll];
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) old[r] = atom_dec_if(d[r] > k, A.deg + u[r], pol);
-            unsigned hm = 0;
+            unsigned hm = 0, nm = 0;
             const int th1 = near_th1(sm);
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
+#if KC_HIT_BF
+                // branch-free outcome; theta crossings (rare) pushed after the loop
+                hm |= (old[r] == k + 1 ? 1u : 0u) << r;
+                lmin = min(lmin, old[r] > k + 1 ? old[r] - 1 : INT_MAX);
+                nm |= (old[r] > k + 1 && old[r] == th1 ? 1u : 0u) << r;
+#else
                 if (old[r] == k + 1) hm |= 1u << r;
                 else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
+#endif
             }
+#if KC_HIT_BF
+            if (nm) {
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++)
+                    if ((nm >> r) & 1u) near_push(A, sm, u[r]);
+            }
+#endif
             const unsigned hb = __ballot_sync(kFull, hm != 0);
             if (lane == 0) PROBE_W(11, (threadIdx.x >> 5) | ((int64_t)__popc(hb) << 8) | ((int64_t)old[0] << 16));
             if (hb) {
@@ -1343,13 +1378,27 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
                 sb1[r] = go ? ld_ro_i64(A.rowptr + u[r] + 1) : 0;
                 old[r] = go ? atom_dec_deg(A.deg + u[r], pol) : INT_MIN;
             }
-            unsigned hm = 0;
+            unsigned hm = 0, nm = 0;
             const int th1 = near_th1(sm);
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
+#if KC_HIT_BF
+                // branch-free outcome; theta crossings (rare) pushed after the loop
+                hm |= (old[r] == k + 1 ? 1u : 0u) << r;
+                lmin = min(lmin, old[r] > k + 1 ? old[r] - 1 : INT_MAX);
+                nm |= (old[r] > k + 1 && old[r] == th1 ? 1u : 0u) << r;
+#else
                 if (old[r] == k + 1) hm |= 1u << r;
                 else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
+#endif
             }
+#if KC_HIT_BF
+            if (nm) {
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++)
+                    if ((nm >> r) & 1u) near_push(A, sm, u[r]);
+            }
+#endif
             if (__any_sync(kFull, hm != 0))
                 handle_hits<true>(A, sm, k, kAsyncNx, u[0], u[1], u[2], u[3], hm, gcnt, nc, sb0, sb1);
         } else {
@@ -1358,13 +1407,27 @@ __device__ int64_t local_drain_async(const KArgs &A, Smem &sm, const int k, bool
                 const int32_t d = u[r] < 0 ? -1 : (atom_only ? INT_MAX : ld_deg(A.deg + u[r], pol));
                 old[r] = atom_dec_if(d > k, A.deg + u[r], pol);
             }
-            unsigned hm = 0;
+            unsigned hm = 0, nm = 0;
             const int th1 = near_th1(sm);
 #pragma unroll
             for (int r = 0; r < kUnroll; r++) {
+#if KC_HIT_BF
+                // branch-free outcome; theta crossings (rare) pushed after the loop
+                hm |= (old[r] == k + 1 ? 1u : 0u) << r;
+                lmin = min(lmin, old[r] > k + 1 ? old[r] - 1 : INT_MAX);
+                nm |= (old[r] > k + 1 && old[r] == th1 ? 1u : 0u) << r;
+#else
                 if (old[r] == k + 1) hm |= 1u << r;
                 else if (old[r] > k + 1) { lmin = min(lmin, old[r] - 1); if (old[r] == th1) near_push(A, sm, u[r]); }
+#endif
             }
+#if KC_HIT_BF
+            if (nm) {
+#pragma unroll
+                for (int r = 0; r < kUnroll; r++)
+                    if ((nm >> r) & 1u) near_push(A, sm, u[r]);
+            }
+#endif
 #ifdef KC_PROBE_W
             {
                 const unsigned hbp = __ballot_sync(kFull, hm != 0);
