@@ -1622,9 +1622,17 @@ __device__ void scan_range(const KArgs &A, const Ctrl &c, Smem &sm, const int32_
             // before this level, so no peel claims it).  Removed vertices left
             // in a lazily compacted list fail the claim.  At k = 0 the frontier
             // is the isolated vertices: nothing walks, nothing races.
+#if KC_HIT_BF
+            // branch-free (an empty slot has vv = dd = -1)
+            const bool live = vv[j] >= 0, shell = live && dd[j] <= k;
+            wm |= (shell ? 1u : 0u) << j;
+            km |= (live && !shell ? 1u : 0u) << j;
+            lmin = min(lmin, live && !shell ? dd[j] : INT_MAX);
+#else
             if (vv[j] < 0) continue;
             if (dd[j] <= k) wm |= 1u << j;
             else { lmin = min(lmin, dd[j]); km |= 1u << j; }
+#endif
         }
         // row bounds of every candidate, in flight together with its claim
         // (at k = 0 every candidate is isolated)
